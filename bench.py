@@ -1,0 +1,297 @@
+#!/usr/bin/env python
+"""bench.py — SPCG iterative phase on B200 (BASELINE.json metric).
+
+Metric: "SPCG iter-phase ms to eps=1e-8 + HBM GB/s per iter vs unsparsified PCG".
+A *step* is one full pass of the hot path: one solve of Algorithm 1 (prologue +
+iterations to ||r|| < 1e-8) on the workload, inputs resident in HBM.  The
+default workload is BASELINE.json configs[1] (C2: 3D 7-point Poisson 64^3,
+ILU(0), SPCG = Algorithm 2 vs PCG = no sparsification).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--sptrsv auto]
+  python bench.py --impl reference ...      # the oracle (plain fp64 C, host cores)
+
+N > 1 (torchrun): every rank solves its own replica of the workload (a single
+system does not shard: DESIGN.md §7), no collective on the data path; times are
+max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import gen  # noqa: E402  (seeded inputs; no method arithmetic)
+
+EPS = 1e-8
+KMAX = 10000
+PAPER_CONTEXT = {"paper_iter_speedup_ilu0_a100_fp32": 1.23, "paper_iter_speedup_iluk_a100_fp32": 1.65,
+                 "paper_e2e_speedup_ilu0_a100_fp32": 1.68, "paper_e2e_speedup_iluk_a100_fp32": 3.73}
+WORKLOADS = {
+    "C1": "C1: 2D 5-point Poisson 32x32 (n=1024), ILU(0)",
+    "C2": "C2: 3D 7-point Poisson 64^3 (n=262144), ILU(0)",
+    "C3": "C3: 3D 27-point Q1 FEM 128^3 (n=2097152), ILU(2)",
+    "C4": "C4: 2D layered anisotropic diffusion 4096^2 (n=16777216), ILU(0)",
+}
+
+
+def _dist():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, burst copy)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def _ncu_traffic(workload: str, impl: str):
+    """dram bytes per launch of the persistent kernel from the committed ncu summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        d = json.load(open(p))
+        e = d.get(workload, {}).get(impl)
+        return None if e is None else float(e["dram_bytes_per_launch"])
+    except Exception:
+        return None
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.path = f"/tmp/spcg_clocks_{os.getpid()}.csv"
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+                 "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+            time.sleep(0.3)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            self.proc.wait()
+
+    def summary(self):
+        try:
+            rows = [l.split(", ") for l in open(self.path).read().strip().splitlines() if l.strip()]
+        except Exception:
+            return None
+        if not rows:
+            return None
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = max(float(r[1]) for r in rows)
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in rows for k in range(4) if len(r) > 4 + k and r[4 + k].strip() == "Active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(rows)}
+
+
+def _cpu_info():
+    model = ""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return model
+
+
+def run_oracle(name: str, A, b, steps: int, warmup: int, budget_s: float = 20.0):
+    """The oracle as it stands (single thread, plain C), timed on the host."""
+    import oracle
+    c = gen.CONFIGS[name]
+    res = {}
+    for mode in ("alg2", "none"):
+        L, U, info = oracle.setup(A, mode=mode, K=c["K"])
+        times, ks = [], []
+        t_start = time.perf_counter()
+        for s in range(warmup + steps):
+            r = oracle.pcg(A, L, U, b, EPS, KMAX)
+            if s >= warmup:
+                times.append(r["seconds"] * 1e3)
+                ks.append(r["k"])
+            if time.perf_counter() - t_start > budget_s and len(times) >= 1:
+                break
+        res[mode] = dict(ms=float(np.mean(times)), k=int(ks[-1]), samples=len(times),
+                         chosen_pct=info["chosen_pct"])
+    return res
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="C2", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="spcg", choices=["spcg", "reference"])
+    ap.add_argument("--sptrsv", default="auto")
+    ap.add_argument("--parts", type=int, default=0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    ws, rank, local = _dist()
+    name = args.workload
+    A = gen.config_matrix(name)
+    b, _ = gen.rhs(A)
+    K = gen.CONFIGS[name]["K"]
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        o = run_oracle(name, A, b, args.steps, args.warmup, budget_s=60.0)
+        v = o["alg2"]["ms"]
+        line = {"metric": "SPCG iter-phase ms to eps=1e-8 + HBM GB/s per iter vs unsparsified PCG",
+                "impl": "reference", "value": v, "unit": "ms", "n_gpus": args.gpus, "steps": o["alg2"]["samples"],
+                "warmup": args.warmup, "ms_per_step": v, "higher_is_better": False, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": WORKLOADS[name], "n": A.n, "nnz": A.nnz, "K": K, "eps": EPS},
+                "iterations": o["alg2"]["k"], "pcg": {"value": o["none"]["ms"], "iterations": o["none"]["k"]},
+                "cpu_baseline": {"value": v, "unit": "ms", "cores": 1, "kind": "oracle",
+                                 "sample": f"full {name} solve to eps=1e-8 (iterative phase only), "
+                                           f"{o['alg2']['samples']} runs, single thread, {_cpu_info()}"},
+                "e2e": {"value": v, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line))
+        return
+
+    import torch
+    import paper_conf_sc_maacsh25_b200 as spcg
+
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl" if torch.cuda.is_available() else "gloo")
+    dev = local if torch.cuda.is_available() else 0
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.current_stream(dev)
+
+    handles = {}
+    for mode in ("alg2", "none"):
+        handles[mode] = spcg.SPCG(A, mode=mode, K=K, sptrsv=args.sptrsv, parts=args.parts, device=dev, stream=stream)
+    bd = torch.from_numpy(b).to(f"cuda:{dev}")
+    xd = torch.empty_like(bd)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=f"cuda:{dev}")
+
+    def barrier():
+        torch.cuda.synchronize(dev)
+        if ws > 1:
+            torch.distributed.barrier()
+            torch.cuda.synchronize(dev)
+
+    results = {}
+    clk = Clocks(dev)
+    with clk:
+        for mode in ("alg2", "none"):
+            h = handles[mode]
+            for _ in range(args.warmup):
+                flush.zero_()
+                h.solve(bd, xd, EPS, KMAX)
+            barrier()
+            ms, ks = [], []
+            t0 = time.perf_counter()
+            for _ in range(args.steps):
+                flush.zero_()                       # L2 flush between steps (256 MiB > 126 MB L2)
+                _, info = h.solve(bd, xd, EPS, KMAX)
+                assert info["status"] == 0, info
+                ms.append(info["iter_phase_ms"])
+                ks.append(info["iterations"])
+            barrier()
+            wall = (time.perf_counter() - t0) * 1e3
+            # e2e through the public API with HOST buffers (H2D b, solve, D2H x inside the call)
+            e2e = []
+            for _ in range(max(3, args.steps // 2)):
+                flush.zero_()
+                torch.cuda.synchronize(dev)
+                te = time.perf_counter()
+                xh, info_h = h.solve_host(b, EPS, KMAX)
+                e2e.append((time.perf_counter() - te) * 1e3)
+            results[mode] = dict(ms=float(np.mean(ms)), ms_max=float(np.max(ms)), k=int(ks[-1]), wall=wall,
+                                 e2e=float(np.mean(e2e)), info=h.info)
+    clocks = clk.summary()
+
+    def mx(v):
+        if ws == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=f"cuda:{dev}")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        return float(t.item())
+
+    s, p = results["alg2"], results["none"]
+    s_ms, p_ms = mx(s["ms"]), mx(p["ms"])
+    s_e2e = mx(s["e2e"])
+    if rank != 0:
+        torch.distributed.destroy_process_group()
+        return
+    peak, peak_src = _peaks()
+    si, pi = s["info"], p["info"]
+    s_bi, p_bi = si["algo_bytes_per_iter"], pi["algo_bytes_per_iter"]
+    s_gbs = s_bi * s["k"] / (s_ms * 1e-3) / 1e9
+    p_gbs = p_bi * p["k"] / (p_ms * 1e-3) / 1e9
+    traffic = _ncu_traffic(name, "spcg")
+    cpu = None
+    if not args.no_cpu_baseline:
+        o = run_oracle(name, A, b, 2, 0, budget_s=20.0)
+        cpu = {"value": o["alg2"]["ms"], "unit": "ms", "cores": 1, "kind": "oracle",
+               "sample": f"full {name} solve to eps=1e-8 (iterative phase), {o['alg2']['samples']} run(s), "
+                         f"single thread, {_cpu_info()}; PCG {o['none']['ms']:.1f} ms"}
+    line = {
+        "metric": "SPCG iter-phase ms to eps=1e-8 + HBM GB/s per iter vs unsparsified PCG",
+        "value": s_ms, "unit": "ms", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": s_ms, "higher_is_better": False, "scaling": "weak", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
+        "config": {"workload": WORKLOADS[name], "n": A.n, "nnz": A.nnz, "K": K, "eps": EPS,
+                   "drop": "Algorithm 2 (tau=1, omega=10%, ratios 10/5/1)", "chosen_pct": si["chosen_pct"],
+                   "sptrsv": si["sptrsv_name"], "ctas": si["parts"],
+                   "l2": "flushed between steps (256 MiB write); timed region = the solve kernel only",
+                   "replicas": ws},
+        "iterations": s["k"], "ms_per_iter": s_ms / max(s["k"], 1),
+        "hbm_gbs_per_iter": s_gbs, "algo_bytes_per_iter": s_bi,
+        "levels": {"L": si["levels_L"], "U": si["levels_U"], "w_A": si["w_A"], "w_Ahat": si["w_Ahat"]},
+        "pcg": {"value": p_ms, "iterations": p["k"], "ms_per_iter": p_ms / max(p["k"], 1), "hbm_gbs_per_iter": p_gbs,
+                "algo_bytes_per_iter": p_bi, "levels": {"L": pi["levels_L"], "U": pi["levels_U"]}},
+        "spcg_vs_pcg": {"iter_phase_speedup": p_ms / s_ms,
+                        "per_iter_speedup": (p_ms / max(p["k"], 1)) / (s_ms / max(s["k"], 1))},
+        "paper_context": PAPER_CONTEXT,
+        "roofline": {"bound": "hbm", "achieved": s_gbs, "peak": peak, "unit": "GB/s", "frac": s_gbs / peak,
+                     "traffic": traffic, "kernel": "spcg_pcg_kernel (persistent, whole Alg. 1)",
+                     "peak_source": peak_src,
+                     "achieved_def": "B_iter (DESIGN.md §4) x iterations / CUDA-event time of the launch"},
+        "cpu_baseline": cpu,
+        "e2e": {"value": s_e2e, "unit": "ms", "h2d_bytes_per_step": 8 * A.n, "d2h_bytes_per_step": 8 * A.n,
+                "path": "spcg_solve with SPCG_HOST_PTRS (pageable host b, x)"},
+        "gpu_launches": args.steps,
+        "clocks": clocks,
+        "setup_ms": {k: si[k] for k in si if k.startswith("setup_ms")},
+    }
+    print(json.dumps(line))
+    if ws > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

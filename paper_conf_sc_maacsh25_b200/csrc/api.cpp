@@ -1,0 +1,315 @@
+// api.cpp — the extern "C" entry points declared in include/spcg.h.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+
+#include "internal.h"
+
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+namespace spcg {
+const char* last_error_cstr();
+}
+
+using namespace spcg;
+
+struct spcg_handle_s {
+    int64_t n = 0;
+    int K = 0;
+    bool identity = false;
+    Csr A;                      // deep copy of the input (device copy lives in dev)
+    SparsifyResult sp;
+    Factors F;
+    Layouts lay;
+    spcg_setup_info_t info{};
+    spcg_device_t* dev = nullptr;
+    int device = -1;
+    std::vector<double> rhist;
+};
+
+template <class T>
+static spcg_status_t put(const std::vector<T>& v, void* buf, size_t* bytes) {
+    size_t need = v.size() * sizeof(T);
+    if (!buf) { *bytes = need; return SPCG_OK; }
+    if (*bytes < need) { set_error("export buffer too small"); return SPCG_ERR_INVALID_ARG; }
+    if (need) std::memcpy(buf, v.data(), need);
+    *bytes = need;
+    return SPCG_OK;
+}
+
+static void level_sets(const std::vector<int32_t>& lev, int64_t w, std::vector<int64_t>& ptr, std::vector<int32_t>& rows) {
+    ptr.assign(w + 1, 0);
+    for (int32_t l : lev) ptr[l + 1]++;
+    for (int64_t l = 0; l < w; ++l) ptr[l + 1] += ptr[l];
+    rows.assign(lev.size(), 0);
+    std::vector<int64_t> nx(ptr.begin(), ptr.end() - 1);
+    for (size_t i = 0; i < lev.size(); ++i) rows[nx[lev[i]]++] = (int32_t)i;
+}
+
+extern "C" {
+
+int32_t spcg_abi_version(void) { return SPCG_ABI_VERSION; }
+
+const char* spcg_status_string(spcg_status_t s) {
+    switch (s) {
+        case SPCG_OK: return "ok";
+        case SPCG_NOT_CONVERGED: return "not converged (x holds x_kmax)";
+        case SPCG_ERR_INVALID_ARG: return "invalid argument";
+        case SPCG_ERR_BAD_MATRIX: return "bad matrix (not square/sorted/symmetric/positive-diagonal/finite)";
+        case SPCG_ERR_ZERO_PIVOT: return "zero or non-finite pivot in ILU";
+        case SPCG_ERR_BREAKDOWN: return "PCG breakdown ((p,w) <= 0 or non-finite scalar)";
+        case SPCG_ERR_OOM: return "out of memory";
+        case SPCG_ERR_CUDA: return "CUDA error";
+        case SPCG_ERR_INTERNAL: return "internal error";
+        case SPCG_ERR_NO_DEVICE: return "handle has no device (host-only setup)";
+        default: return "unknown status";
+    }
+}
+
+const char* spcg_last_error(void) { return last_error_cstr(); }
+
+void spcg_drop_params_default(spcg_drop_params_t* p) {
+    if (!p) return;
+    std::memset(p, 0, sizeof *p);
+    p->mode = SPCG_DROP_WAVEFRONT_AWARE;
+    p->n_ratios = 3;
+    p->ratios_pct[0] = 10.0; p->ratios_pct[1] = 5.0; p->ratios_pct[2] = 1.0;
+    p->tau = 1.0;
+    p->omega_pct = 10.0;
+    p->norm_reading = SPCG_NORM_FRO;
+    p->reduction_denominator = SPCG_DENOM_WA;
+}
+
+void spcg_options_default(spcg_options_t* o) {
+    if (!o) return;
+    std::memset(o, 0, sizeof *o);
+    o->device = 0;
+    o->stream = nullptr;
+    o->sptrsv = SPCG_SPTRSV_AUTO;
+    o->parts = 0;
+    o->host_threads = 0;
+}
+
+int spcg_dev_sm_count(int device);   // kernels.cu
+
+spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_in, int32_t K,
+                         const spcg_options_t* opt_in, spcg_handle_t* out) {
+    if (!out) { set_error("out is NULL"); return SPCG_ERR_INVALID_ARG; }
+    *out = nullptr;
+    if (!Ain || !Ain->row_ptr || (Ain->nnz > 0 && (!Ain->col_idx || !Ain->val))) {
+        set_error("A or its arrays are NULL");
+        return SPCG_ERR_INVALID_ARG;
+    }
+    if (K < -1) { set_error("K must be >= -1"); return SPCG_ERR_INVALID_ARG; }
+    spcg_drop_params_t drop;
+    if (drop_in) drop = *drop_in; else spcg_drop_params_default(&drop);
+    if (drop.mode < 0 || drop.mode > 2) { set_error("bad drop mode"); return SPCG_ERR_INVALID_ARG; }
+    spcg_options_t opt;
+    if (opt_in) opt = *opt_in; else spcg_options_default(&opt);
+#ifdef _OPENMP
+    if (opt.host_threads > 0) omp_set_num_threads(opt.host_threads);
+#endif
+    spcg_handle_s* h = new (std::nothrow) spcg_handle_s();
+    if (!h) return SPCG_ERR_OOM;
+    try {
+        double t0 = now_ms();
+        h->n = Ain->n;
+        h->K = K;
+        h->identity = (K < 0);
+        h->device = opt.device;
+        if (Ain->n <= 0) { delete h; set_error("n must be >= 1"); return SPCG_ERR_INVALID_ARG; }
+        if (Ain->row_ptr[Ain->n] != Ain->nnz) { delete h; set_error("row_ptr[n] != nnz"); return SPCG_ERR_BAD_MATRIX; }
+        h->A.n = Ain->n;
+        h->A.rp.assign(Ain->row_ptr, Ain->row_ptr + Ain->n + 1);
+        h->A.col.assign(Ain->col_idx, Ain->col_idx + Ain->nnz);
+        h->A.val.assign(Ain->val, Ain->val + Ain->nnz);
+        std::vector<int64_t> pos_t;
+        spcg_status_t st = validate_and_mirror(h->A, pos_t);
+        if (st != SPCG_OK) { delete h; return st; }
+        double t1 = now_ms();
+        st = sparsify_select(h->A, pos_t, drop, h->sp);
+        if (st != SPCG_OK) { delete h; return st; }
+        double t2 = now_ms();
+        const Csr& Ah = h->sp.Ahat;
+        st = iluk_symbolic(Ah, K < 0 ? 0 : K, h->F);
+        if (st != SPCG_OK) { delete h; return st; }
+        double t3 = now_ms();
+        st = ilu_numeric(Ah, h->F);
+        h->info.zero_pivot_row = h->F.zero_pivot_row;
+        if (st != SPCG_OK) { delete h; return st; }
+        double t4 = now_ms();
+
+        // executor and grid
+        int sms = 148;
+        if (opt.device >= 0) {
+            sms = spcg_dev_sm_count(opt.device);
+            if (sms <= 0) { delete h; return SPCG_ERR_CUDA; }
+        }
+        int strategy = opt.sptrsv == SPCG_SPTRSV_AUTO ? SPCG_SPTRSV_CHUNKED : opt.sptrsv;
+        if (strategy < 1 || strategy > 3) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }
+        int parts = opt.parts;
+        if (parts <= 0) parts = h->n <= 16384 ? 1 : sms;
+        parts = std::max(1, std::min<int>(parts, sms));
+        if ((int64_t)parts > h->n) parts = (int)h->n;
+        build_spmv_layout(h->A, h->lay.A);
+        build_tri_layouts(h->F, strategy, parts, 16384, h->lay);
+        double t5 = now_ms();
+        int64_t bytes = 0;
+        if (opt.device >= 0) {
+            st = spcg_dev_create(opt.device, opt.stream, h->lay, h->n, h->identity, &h->dev, &bytes);
+            if (st != SPCG_OK) { delete h; return st; }
+        }
+        double t6 = now_ms();
+
+        spcg_setup_info_t& I = h->info;
+        I.chosen_pct = h->sp.chosen_pct;
+        I.m_t = h->sp.m_t;
+        I.w_A = h->sp.w_A;
+        I.w_Ahat = h->sp.w_Ahat;
+        I.n_tried = h->sp.n_tried;
+        for (int r = 0; r < 8; ++r) {
+            I.tried_pct[r] = h->sp.tried_pct[r];
+            I.indicator[r] = h->sp.indicator[r];
+            I.tried_w[r] = h->sp.tried_w[r];
+            I.tried_reduction_pct[r] = h->sp.reduction[r];
+        }
+        I.n = h->n;
+        I.nnz_A = h->A.nnz();
+        I.nnz_Ahat = Ah.nnz();
+        I.nnz_L = h->F.L.nnz();
+        I.nnz_U = h->F.U.nnz();
+        I.levels_L = h->F.wL;
+        I.levels_U = h->F.wU;
+        I.zero_pivot_row = -1;
+        I.setup_ms_validate = t1 - t0;
+        I.setup_ms_sparsify = t2 - t1;
+        I.setup_ms_symbolic = t3 - t2;
+        I.setup_ms_numeric = t4 - t3;
+        I.setup_ms_layout = t5 - t4;
+        I.setup_ms_upload = t6 - t5;
+        I.sptrsv = strategy;
+        I.parts = parts;
+        I.device_bytes = bytes;
+        // B_iter: 12 B per stored entry of A, L_s, U_s; 1/u_ii; three row
+        // pointers; two level_rows arrays; 120 B of vector traffic per row.
+        const double n = (double)h->n;
+        const double nU_s = (double)(I.nnz_U - h->n);
+        if (h->identity) {
+            I.algo_bytes_per_iter = 12.0 * I.nnz_A + 4.0 * (n + 1) + 96.0 * n;
+            I.algo_flops_per_iter = 2.0 * I.nnz_A + 10.0 * n;
+        } else {
+            I.algo_bytes_per_iter = 12.0 * (I.nnz_A + I.nnz_L + nU_s) + 8.0 * n + 12.0 * (n + 1) + 8.0 * n + 120.0 * n;
+            I.algo_flops_per_iter = 2.0 * (I.nnz_A + I.nnz_L + nU_s) + n + 12.0 * n;
+        }
+        *out = h;
+        return SPCG_OK;
+    } catch (const std::bad_alloc&) {
+        delete h;
+        set_error("host allocation failed");
+        return SPCG_ERR_OOM;
+    } catch (...) {
+        delete h;
+        set_error("unexpected exception in setup");
+        return SPCG_ERR_INTERNAL;
+    }
+}
+
+spcg_status_t spcg_get_setup_info(spcg_handle_t h, spcg_setup_info_t* info) {
+    if (!h || !info) return SPCG_ERR_INVALID_ARG;
+    *info = h->info;
+    return SPCG_OK;
+}
+
+spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps, int64_t kmax,
+                         uint32_t flags, spcg_solve_info_t* info) {
+    if (!h || !b || !x || kmax < 0 || !(eps >= 0.0)) { set_error("bad solve arguments"); return SPCG_ERR_INVALID_ARG; }
+    if (!h->dev) { set_error("host-only handle"); return SPCG_ERR_NO_DEVICE; }
+    spcg_solve_info_t tmp{};
+    spcg_solve_info_t* I = info ? info : &tmp;
+    std::memset(I, 0, sizeof *I);
+    try {
+        double t0 = now_ms();
+        spcg_status_t st;
+        if (flags & SPCG_HOST_PTRS) {
+            // host buffers: H2D of b (and x0), solve, D2H of x — all inside the call
+            double* db = nullptr;
+            double* dx = nullptr;
+            st = spcg_dev_copy(h->dev, &db, nullptr, (size_t)h->n * 8, -1);   // alloc
+            if (st != SPCG_OK) return st;
+            st = spcg_dev_copy(h->dev, &dx, nullptr, (size_t)h->n * 8, -1);
+            if (st != SPCG_OK) { spcg_dev_copy(h->dev, db, nullptr, 0, -2); return st; }
+            spcg_dev_copy(h->dev, db, b, (size_t)h->n * 8, 1);
+            if (flags & SPCG_USE_X0) spcg_dev_copy(h->dev, dx, x, (size_t)h->n * 8, 1);
+            st = spcg_dev_solve(h->dev, db, dx, eps, kmax, (flags & SPCG_USE_X0) != 0, I, &h->rhist);
+            spcg_dev_copy(h->dev, x, dx, (size_t)h->n * 8, 2);
+            spcg_dev_copy(h->dev, db, nullptr, 0, -2);
+            spcg_dev_copy(h->dev, dx, nullptr, 0, -2);
+        } else {
+            st = spcg_dev_solve(h->dev, b, x, eps, kmax, (flags & SPCG_USE_X0) != 0, I, &h->rhist);
+        }
+        I->total_ms = now_ms() - t0;
+        return st;
+    } catch (...) {
+        set_error("unexpected exception in solve");
+        return SPCG_ERR_INTERNAL;
+    }
+}
+
+spcg_status_t spcg_apply_spmv(spcg_handle_t h, const double* p, double* w, double* pw) {
+    if (!h || !p || !w) return SPCG_ERR_INVALID_ARG;
+    if (!h->dev) return SPCG_ERR_NO_DEVICE;
+    return spcg_dev_apply(h->dev, 1, p, w, nullptr, pw);
+}
+spcg_status_t spcg_apply_lower(spcg_handle_t h, const double* r, double* y) {
+    if (!h || !r || !y) return SPCG_ERR_INVALID_ARG;
+    if (!h->dev) return SPCG_ERR_NO_DEVICE;
+    return spcg_dev_apply(h->dev, 2, r, y, nullptr, nullptr);
+}
+spcg_status_t spcg_apply_upper(spcg_handle_t h, const double* y, double* z, const double* r, double* rz) {
+    if (!h || !y || !z) return SPCG_ERR_INVALID_ARG;
+    if (!h->dev) return SPCG_ERR_NO_DEVICE;
+    return spcg_dev_apply(h->dev, 3, y, z, r, rz);
+}
+spcg_status_t spcg_apply_precond(spcg_handle_t h, const double* r, double* z, double* rz) {
+    if (!h || !r || !z) return SPCG_ERR_INVALID_ARG;
+    if (!h->dev) return SPCG_ERR_NO_DEVICE;
+    return spcg_dev_apply(h->dev, 4, r, z, r, rz);
+}
+
+spcg_status_t spcg_export(spcg_handle_t h, int32_t what, void* buf, size_t* bytes) {
+    if (!h || !bytes) return SPCG_ERR_INVALID_ARG;
+    const Csr& Ah = h->sp.Ahat;
+    std::vector<int64_t> p64;
+    std::vector<int32_t> r32;
+    switch (what) {
+        case SPCG_EXPORT_AHAT_ROWPTR: return put(Ah.rp, buf, bytes);
+        case SPCG_EXPORT_AHAT_COL: return put(Ah.col, buf, bytes);
+        case SPCG_EXPORT_AHAT_VAL: return put(Ah.val, buf, bytes);
+        case SPCG_EXPORT_L_ROWPTR: return put(h->F.L.rp, buf, bytes);
+        case SPCG_EXPORT_L_COL: return put(h->F.L.col, buf, bytes);
+        case SPCG_EXPORT_L_VAL: return put(h->F.L.val, buf, bytes);
+        case SPCG_EXPORT_U_ROWPTR: return put(h->F.U.rp, buf, bytes);
+        case SPCG_EXPORT_U_COL: return put(h->F.U.col, buf, bytes);
+        case SPCG_EXPORT_U_VAL: return put(h->F.U.val, buf, bytes);
+        case SPCG_EXPORT_FILL_LEVEL: return put(h->F.fill_level, buf, bytes);
+        case SPCG_EXPORT_LEVEL_L: return put(h->F.levL, buf, bytes);
+        case SPCG_EXPORT_LEVEL_U: return put(h->F.levU, buf, bytes);
+        case SPCG_EXPORT_LEVELPTR_L: level_sets(h->F.levL, h->F.wL, p64, r32); return put(p64, buf, bytes);
+        case SPCG_EXPORT_LEVELROWS_L: level_sets(h->F.levL, h->F.wL, p64, r32); return put(r32, buf, bytes);
+        case SPCG_EXPORT_LEVELPTR_U: level_sets(h->F.levU, h->F.wU, p64, r32); return put(p64, buf, bytes);
+        case SPCG_EXPORT_LEVELROWS_U: level_sets(h->F.levU, h->F.wU, p64, r32); return put(r32, buf, bytes);
+        case SPCG_EXPORT_RHIST: return put(h->rhist, buf, bytes);
+        default: set_error("unknown export item"); return SPCG_ERR_INVALID_ARG;
+    }
+}
+
+void spcg_destroy(spcg_handle_t h) {
+    if (!h) return;
+    if (h->dev) spcg_dev_destroy(h->dev);
+    delete h;
+}
+
+}  // extern "C"

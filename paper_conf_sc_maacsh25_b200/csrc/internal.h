@@ -1,0 +1,107 @@
+// internal.h — host-side structures shared by the library's translation units.
+// Not part of the ABI (include/spcg.h is).  No oracle code or header is used here.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/spcg.h"
+
+namespace spcg {
+
+struct Csr {                       // host CSR, int64 row pointers
+    int64_t n = 0;
+    std::vector<int64_t> rp;
+    std::vector<int32_t> col;
+    std::vector<double> val;
+    int64_t nnz() const { return rp.empty() ? 0 : rp.back(); }
+};
+
+void set_error(const std::string& s);
+double now_ms();
+
+// ---- setup.cpp -------------------------------------------------------------
+// Validation (O1 contract) and the transpose map pos_t[q] = position of the
+// mirror entry (j,i) of entry q = (i,j).
+spcg_status_t validate_and_mirror(const Csr& A, std::vector<int64_t>& pos_t);
+
+// Longest-path wavefront levels by Kahn frontier peeling (independent of the
+// oracle's dynamic programme).  lower = true: i depends on j < i in row i;
+// lower = false: i depends on j > i.  Returns number of levels.
+int64_t kahn_levels(const Csr& M, bool lower, std::vector<int32_t>& lev);
+
+struct SparsifyResult {
+    Csr Ahat;
+    double chosen_pct = 0.0;
+    int64_t m_t = 0, w_A = 0, w_Ahat = 0;
+    int n_tried = 0;
+    double tried_pct[8] = {0}, indicator[8] = {0}, reduction[8] = {0};
+    int64_t tried_w[8] = {0};
+};
+spcg_status_t sparsify_select(const Csr& A, const std::vector<int64_t>& pos_t,
+                              const spcg_drop_params_t& p, SparsifyResult& out);
+
+// ILU(K) symbolic by the fill-path characterisation (BFS through lower-numbered
+// vertices), numeric IKJ factorisation (level-parallel over rows).
+struct Factors {
+    Csr L;                         // strictly lower, unit diagonal implicit
+    Csr U;                         // upper incl. diagonal (first in each row)
+    std::vector<int32_t> fill_level;   // per entry of the merged row (L then U), row-major
+    std::vector<int32_t> levL, levU;   // per-row wavefront level of the L / U solve
+    int64_t wL = 0, wU = 0;
+    int64_t zero_pivot_row = -1;
+};
+spcg_status_t iluk_symbolic(const Csr& Ahat, int K, Factors& F);
+spcg_status_t ilu_numeric(const Csr& Ahat, Factors& F);
+
+// ---- layout.cpp ------------------------------------------------------------
+// Sliced-ELL (slice height 32, column-major inside a slice) triangular-solve
+// schedule for one factor.  Entries of slice s occupy [eoff[s]*32, eoff[s+1]*32).
+struct TriLayout {
+    int32_t nslices = 0;
+    std::vector<int64_t> eoff;     // [nslices+1] in units of 32-entry columns
+    std::vector<int32_t> rows;     // [nslices*32], -1 = padding lane
+    std::vector<uint8_t> publish;  // [nslices*32] 1 if the row's value is read through its flag slot
+    std::vector<int32_t> rlen;     // [nslices*32] dependencies of the row (entries beyond are padding)
+    std::vector<int32_t> src;      // [entries*32] >= 0: smem ring slot; < 0: -(j+1) global/flagged
+    std::vector<double> val;       // [entries*32]
+    std::vector<double> dinv;      // [nslices*32] 1/u_ii (upper only)
+    std::vector<int32_t> gptr;     // [ngroups+1] slice ranges of the wavefront groups
+    std::vector<int32_t> part_gptr;// [parts+1]  group ranges per part (chunked); levels: [0, ngroups]
+    int32_t ngroups = 0;
+    int64_t total_cols = 0;        // sum of slice widths
+};
+
+struct SpmvLayout {                // SELL-32 of the original A, natural row order
+    int32_t nslices = 0;
+    std::vector<int64_t> eoff;
+    std::vector<int32_t> col;
+    std::vector<double> val;
+};
+
+struct Layouts {
+    int32_t strategy = SPCG_SPTRSV_LEVEL;
+    int32_t parts = 1;
+    int32_t ring = 0;              // entries of the shared-memory ring (chunked)
+    std::vector<int64_t> part_begin; // [parts+1] contiguous row ranges (chunked)
+    SpmvLayout A;
+    TriLayout L, U;
+};
+
+void build_spmv_layout(const Csr& A, SpmvLayout& out);
+void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, Layouts& out);
+
+}  // namespace spcg
+
+// ---- device side (kernels.cu), plain C++ interface -------------------------
+struct spcg_device_s;
+typedef struct spcg_device_s spcg_device_t;
+
+spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay, int64_t n,
+                              bool identity_precond, spcg_device_t** out, int64_t* bytes);
+void spcg_dev_destroy(spcg_device_t* d);
+spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, double eps, int64_t kmax,
+                             bool use_x0, spcg_solve_info_t* info, std::vector<double>* rhist);
+spcg_status_t spcg_dev_apply(spcg_device_t* d, int op, const double* in, double* out,
+                             const double* aux, double* scalar_out);
+spcg_status_t spcg_dev_copy(spcg_device_t* d, void* dst, const void* src, size_t bytes, int kind);

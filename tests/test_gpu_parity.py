@@ -1,0 +1,149 @@
+"""CUDA path (through the C ABI) vs the oracle, element by element, on seeded
+inputs.  Tolerances: SpMV / SpTRSV <= 1e-12 relative to the
+row's absolute sum of terms; PCG |k_gpu - k_oracle| <= 1 on convergence runs and
+||x_gpu - x_oracle|| <= 1e-8 ||x_oracle|| in forced-k runs (eps = 0, kmax = k)."""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+import paper_conf_sc_maacsh25_b200 as lib
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+EXECUTORS = ["level", "syncfree", "chunked"]
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, np.float64)).cuda()
+
+
+def _csr_abs(M):
+    return gen.CSR(M.n, M.row_ptr, M.col, np.abs(M.val))
+
+
+# sizes: several 32-row slices, a ragged tail, more rows than one CTA's block
+SMALL = [("poisson2d", (37, 29), 0), ("poisson3d", (13, 11, 9), 0), ("fem_q1", (9, 8, 7, 3), 2),
+         ("aniso_layered", (150, 67, 4), 0)]
+
+
+@pytest.mark.parametrize("fam,params,K", SMALL)
+@pytest.mark.parametrize("ex", EXECUTORS)
+@pytest.mark.parametrize("parts", [1, 7, 0])
+def test_operators_match_oracle(fam, params, K, ex, parts):
+    A = gen.make(fam, *params)
+    h = lib.SPCG(A, mode="alg2", K=K, sptrsv=ex, parts=parts)
+    L, U, _ = oracle.setup(A, mode="alg2", K=K)
+    rng = np.random.default_rng(5)
+    p = rng.standard_normal(A.n)
+    # SpMV w = A p and (p, w)
+    w = torch.zeros(A.n, dtype=torch.float64, device="cuda")
+    pw = h.apply_spmv(_dev(p), w)
+    wr = oracle.spmv(A, p)
+    scale = oracle.spmv(_csr_abs(A), np.abs(p)) + 1e-300
+    assert np.all(np.abs(w.cpu().numpy() - wr) <= 1e-13 * scale)
+    assert pw == pytest.approx(float(np.dot(p, wr)), rel=1e-12)
+    # forward solve y = L^-1 r
+    r = rng.standard_normal(A.n)
+    y = torch.zeros_like(w)
+    h.apply_lower(_dev(r), y)
+    yr = oracle.sptrsv_lower(L, r)
+    assert np.allclose(y.cpu().numpy(), yr, rtol=1e-12, atol=1e-12 * np.abs(yr).max())
+    # backward solve z = U^-1 y with (r, z)
+    z = torch.zeros_like(w)
+    rz = h.apply_upper(_dev(yr), z, _dev(r))
+    zr = oracle.sptrsv_upper(U, yr)
+    assert np.allclose(z.cpu().numpy(), zr, rtol=1e-12, atol=1e-12 * np.abs(zr).max())
+    assert rz == pytest.approx(float(np.dot(r, zr)), rel=1e-11)
+    # whole preconditioner
+    z2 = torch.zeros_like(w)
+    h.apply_precond(_dev(r), z2)
+    assert np.allclose(z2.cpu().numpy(), zr, rtol=1e-12, atol=1e-12 * np.abs(zr).max())
+    h.close()
+
+
+@pytest.mark.parametrize("fam,params,K", SMALL + [("poisson2d", (32, 32), 0)])
+@pytest.mark.parametrize("mode", ["alg2", "none"])
+@pytest.mark.parametrize("ex", EXECUTORS)
+def test_pcg_matches_oracle(fam, params, K, mode, ex):
+    A = gen.make(fam, *params)
+    b, xt = gen.rhs(A)
+    h = lib.SPCG(A, mode=mode, K=K, sptrsv=ex)
+    L, U, _ = oracle.setup(A, mode=mode, K=K)
+    ro = oracle.pcg(A, L, U, b, 1e-8, 5000)
+    x, info = h.solve(_dev(b), eps=1e-8, kmax=5000)
+    assert info["status"] == 0 and info["converged"]
+    assert abs(info["iterations"] - ro["k"]) <= 1
+    # true residual of the GPU solution
+    xg = x.cpu().numpy()
+    assert np.linalg.norm(b - oracle.spmv(A, xg)) <= 1.01e-8 * 1.5
+    # forced-k: same number of iterations, solution within 1e-8 (expect ~1e-13)
+    k = ro["k"]
+    xf, inf2 = h.solve(_dev(b), eps=0.0, kmax=k)
+    assert inf2["iterations"] == k and inf2["status"] == 0
+    rel = np.linalg.norm(xf.cpu().numpy() - ro["x"]) / np.linalg.norm(ro["x"])
+    assert rel <= 1e-8, rel
+    # residual history agrees with the oracle's
+    rh = h.rhist()
+    assert len(rh) == k + 1
+    assert np.allclose(rh, ro["rhist"], rtol=1e-6, atol=1e-14)
+    h.close()
+
+
+def test_identity_preconditioner_is_cg():
+    A = gen.make("poisson2d", 40, 23)
+    b, _ = gen.rhs(A)
+    h = lib.SPCG(A, mode="none", K=-1)
+    ro = oracle.pcg(A, None, None, b, 1e-8, 5000)
+    x, info = h.solve(_dev(b), eps=1e-8, kmax=5000)
+    assert abs(info["iterations"] - ro["k"]) <= 1
+    xf, _ = h.solve(_dev(b), eps=0.0, kmax=ro["k"])
+    assert np.linalg.norm(xf.cpu().numpy() - ro["x"]) <= 1e-8 * np.linalg.norm(ro["x"])
+
+
+@pytest.mark.parametrize("ex", EXECUTORS)
+def test_deterministic_bitwise(ex):
+    A = gen.make("aniso_layered", 300, 211, 4)
+    b, _ = gen.rhs(A)
+    h = lib.SPCG(A, sptrsv=ex)
+    x1, i1 = h.solve(_dev(b), eps=1e-8, kmax=5000)
+    x2, i2 = h.solve(_dev(b), eps=1e-8, kmax=5000)
+    assert i1["iterations"] == i2["iterations"]
+    assert torch.equal(x1, x2)
+
+
+def test_host_pointer_path_matches_device_path():
+    A = gen.make("poisson3d", 20, 20, 20)
+    b, _ = gen.rhs(A)
+    h = lib.SPCG(A)
+    xd, i1 = h.solve(_dev(b), eps=1e-8, kmax=5000)
+    xh, i2 = h.solve_host(b, eps=1e-8, kmax=5000)
+    assert i1["iterations"] == i2["iterations"]
+    assert np.array_equal(xd.cpu().numpy(), xh)
+
+
+def test_initial_guess_and_kmax():
+    A = gen.make("poisson2d", 33, 31)
+    b, xt = gen.rhs(A)
+    h = lib.SPCG(A)
+    L, U, _ = oracle.setup(A, mode="alg2", K=0)
+    x0 = 0.5 * xt
+    ro = oracle.pcg(A, L, U, b, 0.0, 6, x0=x0)
+    xg = _dev(x0)
+    h.solve(_dev(b), xg, eps=0.0, kmax=6, use_x0=True)
+    assert np.linalg.norm(xg.cpu().numpy() - ro["x"]) <= 1e-10 * np.linalg.norm(ro["x"])
+    x, info = h.solve(_dev(b), eps=1e-30, kmax=4)
+    assert info["iterations"] == 4 and info["status"] == lib.NOT_CONVERGED
+
+
+def test_tridiagonal_one_iteration():
+    n = 1000
+    d = np.zeros((n, n))
+    A = gen.from_dense(np.diag(np.full(n, 2.5)) + np.diag(np.full(n - 1, -1.0), 1) + np.diag(np.full(n - 1, -1.0), -1))
+    b, _ = gen.rhs(A)
+    for ex in EXECUTORS:
+        h = lib.SPCG(A, mode="none", sptrsv=ex, parts=4)
+        x, info = h.solve(_dev(b), eps=1e-12, kmax=50)
+        assert info["iterations"] == 1, ex       # ILU(0) of a tridiagonal matrix is exact (P8)
+        h.close()
