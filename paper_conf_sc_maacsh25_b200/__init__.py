@@ -33,11 +33,13 @@ USE_X0, HOST_PTRS = 0x1, 0x2
 
 EXPORT = dict(ahat_rowptr=1, ahat_col=2, ahat_val=3, l_rowptr=4, l_col=5, l_val=6, u_rowptr=7, u_col=8,
               u_val=9, fill_level=10, level_l=11, level_u=12, levelptr_l=13, levelrows_l=14,
-              levelptr_u=15, levelrows_u=16, rhist=17)
+              levelptr_u=15, levelrows_u=16, rhist=17, dbg_stream=100, dbg_part_chunk=101, dbg_part_uchunk=102,
+              dbg_part_begin=103)
 _EXPORT_DT = dict(ahat_rowptr=np.int64, ahat_col=np.int32, ahat_val=np.float64, l_rowptr=np.int64,
                   l_col=np.int32, l_val=np.float64, u_rowptr=np.int64, u_col=np.int32, u_val=np.float64,
                   fill_level=np.int32, level_l=np.int32, level_u=np.int32, levelptr_l=np.int64,
-                  levelrows_l=np.int32, levelptr_u=np.int64, levelrows_u=np.int32, rhist=np.float64)
+                  levelrows_l=np.int32, levelptr_u=np.int64, levelrows_u=np.int32, rhist=np.float64,
+                  dbg_stream=np.uint8, dbg_part_chunk=np.int32, dbg_part_uchunk=np.int32, dbg_part_begin=np.int64)
 
 
 class SpcgError(RuntimeError):
@@ -190,9 +192,13 @@ class SPCG:
         self.info["sptrsv_name"] = SPTRSV_NAME.get(self.info["sptrsv"], "?")
 
     def close(self):
-        if getattr(self, "_h", None):
-            load().spcg_destroy(self._h)
-            self._h = None
+        h = getattr(self, "_h", None)
+        self._h = None
+        if h and _lib is not None:
+            try:
+                _lib.spcg_destroy(h)
+            except Exception:      # interpreter shutdown
+                pass
 
     __del__ = close
 

@@ -302,8 +302,19 @@ spcg_status_t spcg_export(spcg_handle_t h, int32_t what, void* buf, size_t* byte
         case SPCG_EXPORT_LEVELPTR_U: level_sets(h->F.levU, h->F.wU, p64, r32); return put(p64, buf, bytes);
         case SPCG_EXPORT_LEVELROWS_U: level_sets(h->F.levU, h->F.wU, p64, r32); return put(r32, buf, bytes);
         case SPCG_EXPORT_RHIST: return put(h->rhist, buf, bytes);
+        case 100: return put(h->lay.S.bytes, buf, bytes);          // debug: chunked record stream
+        case 101: return put(h->lay.S.part_chunk, buf, bytes);
+        case 102: return put(h->lay.S.part_uchunk, buf, bytes);
+        case 103: return put(h->lay.part_begin, buf, bytes);
         default: set_error("unknown export item"); return SPCG_ERR_INVALID_ARG;
     }
+}
+
+// debug only (not in spcg.h): heartbeat snapshot of a possibly running solve
+int spcg_dbg_heartbeats(void* dev, unsigned long long* out, int n);
+int spcg_dbg_handle_heartbeats(spcg_handle_t h, unsigned long long* out, int n) {
+    if (!h || !h->dev) return -1;
+    return spcg_dbg_heartbeats((void*)h->dev, out, n);
 }
 
 void spcg_destroy(spcg_handle_t h) {

@@ -79,6 +79,27 @@ struct SpmvLayout {                // SELL-32 of the original A, natural row ord
     std::vector<double> val;
 };
 
+// Chunked executor stream.  Per part (CTA) one byte stream of
+// slice records, L section then U section, cut into CHUNK-byte chunks that the
+// kernel copies into a shared-memory ring with cp.async.bulk.
+constexpr int SPCG_CHUNK_BYTES = 4096;
+constexpr int SPCG_NCHUNK = 8;          // ring slots
+constexpr int SPCG_MAXREC = 8;          // records per chunk (side-data slots)
+constexpr int SPCG_WCAP = 8;            // entry columns per record
+constexpr int SPCG_NSOLVER = 1;         // solver warps per CTA (one software-pipelined chain)
+constexpr int SPCG_REC_HDR = 272;       // 16 B header + 32 x {int32 row, uint32 meta}
+enum { REC_FIRST = 1, REC_LAST = 2, REC_SYNC = 4, REC_UPPER = 8, REC_EXT = 16, REC_WIDE = 32 };
+constexpr int SPCG_WP = 4;              // entry columns the pipelined solver keeps in registers
+
+struct ChunkStream {
+    std::vector<uint8_t> bytes;          // nchunks * CHUNK_BYTES
+    std::vector<int32_t> part_chunk;     // [parts+1] first chunk of each part
+    std::vector<int32_t> part_uchunk;    // [parts]   first U chunk of each part
+    std::vector<uint32_t> chunk_bytes;   // [nchunks]  used bytes (what the bulk copy moves)
+    int64_t used_bytes = 0;
+    int64_t records = 0;
+};
+
 struct Layouts {
     int32_t strategy = SPCG_SPTRSV_LEVEL;
     int32_t parts = 1;
@@ -86,6 +107,7 @@ struct Layouts {
     std::vector<int64_t> part_begin; // [parts+1] contiguous row ranges (chunked)
     SpmvLayout A;
     TriLayout L, U;
+    ChunkStream S;                 // chunked executor only
 };
 
 void build_spmv_layout(const Csr& A, SpmvLayout& out);

@@ -27,16 +27,19 @@
 
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
 #include "internal.h"
 
+using namespace spcg;
+
 namespace {
 
-constexpr int BLOCK = 512;
+constexpr int BLOCK = 384;
 constexpr int NWARP = BLOCK / 32;
-constexpr unsigned long long SPIN_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;   // 20 s: abort, never hang
+constexpr long long SPIN_TIMEOUT_CYC = 8ll * 1000 * 1000 * 1000;            // ~4 s of SM cycles: abort, never hang
 
 enum { ST_LEVEL = SPCG_SPTRSV_LEVEL, ST_SYNCFREE = SPCG_SPTRSV_SYNCFREE, ST_CHUNKED = SPCG_SPTRSV_CHUNKED };
 enum { K_APPLY = 0, K_PRO = 1, K_ITER = 2 };
@@ -85,6 +88,10 @@ struct Params {
     DevA A;
     DevTri L, U;
     const int64_t* part_begin;
+    const uint8_t* stream;         // chunked executor: record stream (SPCG_CHUNK_BYTES per chunk)
+    const int32_t* part_chunk;     // [parts+1]
+    const int32_t* part_uchunk;    // [parts]
+    const unsigned* chunk_bytes;   // used bytes of every chunk
     const double* b;
     double* x;
     double* r;
@@ -101,7 +108,39 @@ struct Params {
     Scal* sc;
     double* rhist;
     long long rhist_cap;
+    unsigned long long* trace;     // debug timeline (env SPCG_TRACE), see trace_mark
+    unsigned long long* hb;        // debug heartbeats [parts][8] (env SPCG_TRACE), see hbeat
 };
+// heartbeat: role slot of this CTA <- (iteration << 40) | (phase step << 20) | value
+__device__ __forceinline__ void hbeat(const Params& P, int role, unsigned long long v) {
+    if (P.hb) *(volatile unsigned long long*)(P.hb + 8 * blockIdx.x + role) = v;
+}
+
+// Debug timeline: globaltimer stamps of iteration TRACE_IT.  [0..7] CTA 0 phase
+// boundaries; [8 + 4c + e] per-CTA solver events (e: 0 first L record, 1 L done,
+// 2 U done, 3 phase end).
+constexpr int TRACE_IT = 2;
+__device__ __forceinline__ void trace_max(const Params& P, long long k, int idx) {
+    if (P.trace && k == TRACE_IT && blockIdx.x == 0 && idx < 400) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        atomicMax(P.trace + 8 + 4 * gridDim.x + idx, t);
+    }
+}
+__device__ __forceinline__ void trace_x(const Params& P, long long k, int idx) {
+    if (P.trace && k == TRACE_IT && blockIdx.x == 0 && idx < 400) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        P.trace[8 + 4 * gridDim.x + idx] = t;
+    }
+}
+__device__ __forceinline__ void trace_mark(const Params& P, long long k, int idx) {
+    if (P.trace && k == TRACE_IT) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        P.trace[idx] = t;
+    }
+}
 
 // ------------------------------------------------------------------ primitives
 __device__ __forceinline__ unsigned long long gtimer() {
@@ -131,7 +170,7 @@ __device__ __forceinline__ void ll_store(uint4* p, double v, unsigned ep) {
 }
 
 __device__ __noinline__ double ll_wait_slow(const uint4* p, unsigned ep, Scal* sc) {
-    unsigned long long t0 = gtimer();
+    const long long t0 = clock64();
     unsigned a, e1, c, e2;
     for (;;) {
         asm volatile("ld.volatile.global.v4.u32 {%0, %1, %2, %3}, [%4];"
@@ -140,7 +179,7 @@ __device__ __noinline__ double ll_wait_slow(const uint4* p, unsigned ep, Scal* s
                      : "memory");
         if (e1 == ep && e2 == ep) break;
         if (ld_volatile_int(&sc->abort)) return 0.0;
-        if (gtimer() - t0 > SPIN_TIMEOUT_NS) {
+        if (clock64() - t0 > SPIN_TIMEOUT_CYC) {
             if (atomicExch(&sc->abort, 1) == 0) {
                 sc->dbg_addr = (long long)(size_t)p;
                 sc->dbg_want = ep;
@@ -175,10 +214,10 @@ __device__ __forceinline__ void grid_sync(Scal* sc, unsigned& gen) {
                 __threadfence();
                 st_release_u32(&sc->bar_gen, g + 1);
             } else {
-                unsigned long long t0 = gtimer();
+                const long long t0 = clock64();
                 while (ld_acquire_u32(&sc->bar_gen) == g) {
                     if (ld_volatile_int(&sc->abort)) break;
-                    if (gtimer() - t0 > SPIN_TIMEOUT_NS) { atomicExch(&sc->abort, 1); break; }
+                    if (clock64() - t0 > SPIN_TIMEOUT_CYC) { atomicExch(&sc->abort, 1); break; }
                 }
             }
             gen = g + 1;
@@ -333,18 +372,562 @@ __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const doub
         const int64_t W = (int64_t)gridDim.x * NWARP;
         for (int64_t s = (int64_t)blockIdx.x * NWARP + warp; s < T.nslices; s += W)
             tri_slice<STRAT, UPPER>(P, T, s, kind, in, out, rdot, mb, ep, alpha, acc_dot, ring, 0, 0);
-    } else {
-        const int c = blockIdx.x;
-        const int64_t pb = P.part_begin[c];
-        const int mask = P.ring - 1;
-        const int g0 = __ldg(T.part_gptr + c), g1 = __ldg(T.part_gptr + c + 1);
-        for (int g = g0; g < g1; ++g) {
-            const int s0 = __ldg(T.gptr + g), s1 = __ldg(T.gptr + g + 1);
-            for (int s = s0 + warp; s < s1; s += NWARP)
-                tri_slice<STRAT, UPPER>(P, T, s, kind, in, out, rdot, mb, ep, alpha, acc_dot, ring, pb, mask);
-            __syncthreads();
+    }
+}
+
+// ------------------------------------------------------------------ chunked pipeline
+// Warp roles inside a CTA during a triangular-solve phase:
+//   warp 0        producer: one lane streams the part's record chunks into the
+//                 shared-memory ring with cp.async.bulk (TMA), mbarrier complete_tx
+//   warp 1        poller: a few records ahead of the solvers, polls the ready flags
+//                 of cross-CTA dependencies and leaves their partial sum in smem
+//   warps 2..10   vector warps: per record, the dynamic per-row operands (fused
+//                 x/r update and ||r||^2 for L; y_i and r_i for U)
+//   warp 11       solver warp: the dependency chain, software-pipelined one record
+//                 ahead so only ring gather -> FMA -> store sits on the critical path
+constexpr int PRODUCER_WARP = 0;
+constexpr int POLLER_WARP = 1;
+constexpr int VEC_WARP0 = 2;
+constexpr int NVEC = 9;
+constexpr int SOLVER_WARP0 = VEC_WARP0 + NVEC;
+static_assert(SOLVER_WARP0 + SPCG_NSOLVER == NWARP, "warp roles must fill the CTA");
+constexpr int POLL_AHEAD = 8;                     // records
+constexpr int SIDE_BYTES = 3 * 256 + 16;          // vec[32], aux[32], ext[32], ext mask
+constexpr size_t CH_RING_BYTES = (size_t)SPCG_NCHUNK * SPCG_CHUNK_BYTES;
+constexpr size_t CH_SIDE_BYTES = (size_t)SPCG_NCHUNK * SPCG_MAXREC * SIDE_BYTES;
+constexpr size_t CH_BAR_BYTES = 512;
+
+__host__ __device__ constexpr size_t chunked_smem_bytes(int ring) {
+    return (size_t)ring * 8 + CH_RING_BYTES + CH_SIDE_BYTES + CH_BAR_BYTES;
+}
+
+struct ChunkSmem {
+    double* yring;
+    uint8_t* chunks;
+    uint8_t* side;
+    uint64_t* full;        // [NCHUNK] TMA landed
+    uint64_t* vfull;       // [NCHUNK] vector operands filled
+    uint64_t* empty;       // [NCHUNK] solvers + poller done
+    uint64_t* ldone;       // solvers finished the L section
+    volatile long long* progress;   // [NSOLVER] record index each solver warp is at
+};
+
+struct PipeState {         // identical sequence in every role
+    unsigned q;            // chunks consumed in this launch
+    unsigned ldone_uses;
+    long long rec;         // records walked in this launch
+    long long k;           // iteration (debug timeline only)
+};
+
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* b, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* b, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
+    unsigned ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(b)), "r"(parity), "r"(20000u)   // suspend (HW sleep) until the phase completes (<= 20 us)
+        : "memory");
+    return ok != 0;
+}
+__device__ __noinline__ void mbar_wait_slow(uint64_t* b, unsigned parity, Scal* sc) {
+    const long long t0 = clock64();
+    unsigned it = 0;
+    while (!mbar_try(b, parity)) {
+        if ((++it & 3) == 0) {
+            if (ld_volatile_int(&sc->abort)) return;
+            if (clock64() - t0 > SPIN_TIMEOUT_CYC) { atomicExch(&sc->abort, 1); return; }
         }
     }
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity, Scal* sc) {
+    if (!mbar_try(b, parity)) mbar_wait_slow(b, parity, sc);
+}
+// After an abort the ring may hold stale chunks: roles must stop parsing them.
+// Warp-collective code must take this decision warp-uniformly (a per-lane read
+// of a racy flag lets lanes disagree; a divergent break then deadlocks the
+// warp at its next __syncwarp / shuffle).
+__device__ __forceinline__ bool aborted(Scal* sc) {
+    return __any_sync(0xffffffffu, ld_volatile_int(&sc->abort) != 0);
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
+__device__ ChunkSmem chunk_smem(double* dyn, int ring) {
+    ChunkSmem S;
+    uint8_t* base = (uint8_t*)dyn;
+    S.yring = dyn;
+    S.chunks = base + (size_t)ring * 8;
+    S.side = S.chunks + CH_RING_BYTES;
+    uint64_t* bars = (uint64_t*)(S.side + CH_SIDE_BYTES);
+    S.full = bars;
+    S.vfull = bars + SPCG_NCHUNK;
+    S.empty = bars + 2 * SPCG_NCHUNK;
+    S.ldone = bars + 3 * SPCG_NCHUNK;
+    S.progress = (volatile long long*)(bars + 3 * SPCG_NCHUNK + 1);
+    return S;
+}
+
+__device__ void chunk_init(const ChunkSmem& S) {
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < SPCG_NCHUNK; ++i) {
+            mbar_init(&S.full[i], 1);
+            mbar_init(&S.vfull[i], NVEC);
+            mbar_init(&S.empty[i], SPCG_NSOLVER + 1);
+        }
+        mbar_init(S.ldone, SPCG_NSOLVER);
+        for (int i = 0; i < SPCG_NSOLVER; ++i) S.progress[i] = -1;
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+}
+
+// record view (byte layout written by layout.cpp emit_section):
+//   [0,16)    header {u16 w, u16 flags, u8 warp, u8 side, u16 bytes, u32 publish, u32 active}
+//   [16,272)  32 lane words {int32 row, u32 meta = len | ne << 8 | publish << 16}
+//   [272, +128w) int32 src[w][32]; then f64 val[w][32]; then f64 dinv[32] (U, LAST)
+struct Rec {
+    const uint8_t* p;
+    uint4 h;
+    __device__ __forceinline__ explicit Rec(const uint8_t* q) : p(q), h(*(const uint4*)q) {}
+    __device__ __forceinline__ int w() const { return (int)(h.x & 0xffffu); }
+    __device__ __forceinline__ int flags() const { return (int)(h.x >> 16); }
+    __device__ __forceinline__ int warp() const { return (int)(h.y & 0xffu); }
+    __device__ __forceinline__ int bytes() const { return (int)(h.y >> 16); }
+    __device__ __forceinline__ int2 lane(int l) const { return *(const int2*)(p + 16 + 8 * l); }
+    __device__ __forceinline__ int row(int l) const { return *(const int*)(p + 16 + 8 * l); }
+    __device__ __forceinline__ int src(int k, int l) const { return *(const int32_t*)(p + SPCG_REC_HDR + 128 * k + 4 * l); }
+    __device__ __forceinline__ double val(int k, int l) const {
+        return *(const double*)(p + SPCG_REC_HDR + 128 * w() + 256 * k + 8 * l);
+    }
+    __device__ __forceinline__ double dinv(int l) const { return *(const double*)(p + SPCG_REC_HDR + 384 * w() + 8 * l); }
+};
+__device__ __forceinline__ int meta_len(unsigned m) { return (int)(m & 0xffu); }
+__device__ __forceinline__ int meta_ne(unsigned m) { return (int)((m >> 8) & 0xffu); }
+__device__ __forceinline__ bool meta_pub(unsigned m) { return (m >> 16) & 1u; }
+__device__ __forceinline__ double* side_vec(const ChunkSmem& S, int slot, int r) {
+    return (double*)(S.side + ((size_t)slot * SPCG_MAXREC + r) * SIDE_BYTES);
+}
+__device__ __forceinline__ double* side_aux(const ChunkSmem& S, int slot, int r) { return side_vec(S, slot, r) + 32; }
+__device__ __forceinline__ double* side_ext(const ChunkSmem& S, int slot, int r) { return side_vec(S, slot, r) + 64; }
+__device__ __forceinline__ unsigned* side_mask(const ChunkSmem& S, int slot, int r) {
+    return (unsigned*)(side_vec(S, slot, r) + 96);
+}
+
+// sum of the leading ne external terms v_k * y_k (k order), polling the flags in one batch
+__device__ __forceinline__ bool ext_try(const Rec& R, int lane, int ne, const uint4* mb, unsigned ep, double& out) {
+    double acc = 0.0;
+    bool ok = true;
+    for (int k0 = 0; k0 < ne; k0 += 4) {
+        uint4 v[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t)
+            if (k0 + t < ne) {
+                const uint4* a = mb + (-R.src(k0 + t, lane) - 1);
+                asm volatile("ld.volatile.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                             : "=r"(v[t].x), "=r"(v[t].y), "=r"(v[t].z), "=r"(v[t].w)
+                             : "l"(a)
+                             : "memory");
+            }
+#pragma unroll
+        for (int t = 0; t < 4; ++t)
+            if (k0 + t < ne) {
+                if (v[t].y != ep || v[t].w != ep) ok = false;
+                const double y = __longlong_as_double((long long)(((unsigned long long)v[t].z << 32) | v[t].x));
+                acc = fma(R.val(k0 + t, lane), y, acc);
+            }
+    }
+    out = acc;
+    return ok;
+}
+
+__device__ double ext_wait(const Rec& R, int lane, int ne, const uint4* mb, unsigned ep, Scal* sc) {
+    double acc;
+    if (ext_try(R, lane, ne, mb, ep, acc)) return acc;
+    acc = 0.0;
+    for (int k = 0; k < ne; ++k) acc = fma(R.val(k, lane), ll_wait(mb + (-R.src(k, lane) - 1), ep, sc), acc);
+    return acc;
+}
+
+// ring part of a record for a compile-time width W (warp-uniform dispatch keeps
+// the instruction count proportional to the record's real width)
+template <int W>
+__device__ __forceinline__ double ring_terms(const uint8_t* p, int lane, int ne, int len, const double* yring,
+                                             double acc) {
+    const uint8_t* sp = p + SPCG_REC_HDR + 4 * lane;
+    const uint8_t* vp = p + SPCG_REC_HDR + 128 * W + 8 * lane;
+    int sidx[W > 0 ? W : 1];
+    double v[W > 0 ? W : 1], d[W > 0 ? W : 1];
+#pragma unroll
+    for (int k = 0; k < W; ++k) {
+        const bool on = k >= ne && k < len;
+        sidx[k] = on ? *(const int*)(sp + 128 * k) : 0;
+        v[k] = on ? *(const double*)(vp + 256 * k) : 0.0;
+    }
+#pragma unroll
+    for (int k = 0; k < W; ++k) d[k] = yring[sidx[k]];
+#pragma unroll
+    for (int k = 0; k < W; ++k) acc = fma(-v[k], d[k], acc);   // v = 0 for masked-off k: acc unchanged
+    return acc;
+}
+
+__device__ __forceinline__ double ring_terms_dispatch(int wd, const uint8_t* p, int lane, int ne, int len,
+                                                      const double* yring, double acc) {
+    switch (wd) {
+        case 0: return acc;
+        case 1: return ring_terms<1>(p, lane, ne, len, yring, acc);
+        case 2: return ring_terms<2>(p, lane, ne, len, yring, acc);
+        case 3: return ring_terms<3>(p, lane, ne, len, yring, acc);
+        case 4: return ring_terms<4>(p, lane, ne, len, yring, acc);
+        case 5: return ring_terms<5>(p, lane, ne, len, yring, acc);
+        case 6: return ring_terms<6>(p, lane, ne, len, yring, acc);
+        case 7: return ring_terms<7>(p, lane, ne, len, yring, acc);
+        default: return ring_terms<8>(p, lane, ne, len, yring, acc);
+    }
+}
+
+// One record's operands as held in registers by the pipelined solver warp.
+constexpr int WP = SPCG_WP;
+struct Bundle {
+    const uint8_t* p;
+    int fl, slot, r, row;
+    unsigned meta;
+    double vec, dinv, aux;
+    int sidx[WP];
+    double v[WP];
+};
+
+template <bool UPPER>
+__device__ __forceinline__ void bundle_load(Bundle& B, const ChunkSmem& S, const uint8_t* p, int slot, int r, int lane) {
+    B.p = p;
+    B.slot = slot;
+    B.r = r;
+    const uint4 h = *(const uint4*)p;
+    B.fl = (int)(h.x >> 16);
+    const int wd = (int)(h.x & 0xffffu);
+    const int2 lw = *(const int2*)(p + 16 + 8 * lane);
+    B.row = lw.x;
+    B.meta = (unsigned)lw.y;
+    const int len = meta_len(B.meta), ne = meta_ne(B.meta);
+    const uint8_t* sp = p + SPCG_REC_HDR + 4 * lane;
+    const uint8_t* vp = p + SPCG_REC_HDR + 128 * wd + 8 * lane;
+#pragma unroll
+    for (int k = 0; k < WP; ++k) {
+        const bool on = k >= ne && k < len && k < wd;      // ring entries only
+        B.sidx[k] = on ? *(const int*)(sp + 128 * k) : 0;
+        B.v[k] = on ? *(const double*)(vp + 256 * k) : 0.0;
+    }
+    B.vec = side_vec(S, slot, r)[lane];                     // meaningful on FIRST records
+    if (UPPER) {
+        B.dinv = (B.fl & REC_LAST) ? *(const double*)(p + SPCG_REC_HDR + 384 * wd + 8 * lane) : 1.0;
+        B.aux = side_aux(S, slot, r)[lane];
+    }
+}
+
+// The solver warp over one section (all L records or all U records of the part),
+// software-pipelined one record deep: while record t computes, record t+1's
+// header, lane word, entries and side operands are already in registers, so
+// only ring gather -> FMA chain -> ring store is on the dependency path.
+template <bool UPPER, bool PRO>
+__device__ __noinline__ void solver_section(const Params& P, const ChunkSmem& S, unsigned q0, int ib, int ie,
+                                            long long recn, double* out, const double* rdot, const uint4* mb,
+                                            unsigned ep, int64_t pb, int mask, double* rz_io) {
+    const int lane = threadIdx.x & 31;
+    double rz = *rz_io;
+    double acc_carry = 0.0;          // accumulator of a row continued in the next record
+    // open the first chunk that has records (empty chunks are released at once)
+    int i = ib, nrec = 0, slot = 0;
+    const uint8_t* rp = nullptr;
+    for (;;) {
+        const unsigned q = q0 + i;
+        slot = q % SPCG_NCHUNK;
+        mbar_wait(&S.vfull[slot], (q / SPCG_NCHUNK) & 1, P.sc);
+        if (aborted(P.sc)) { *rz_io = rz; return; }
+        const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
+        nrec = *(const uint16_t*)ch;
+        rp = ch + 16;
+        if (nrec > 0) break;
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&S.empty[slot]);
+        if (++i >= ie) { *rz_io = rz; return; }
+    }
+    int r = 0;
+    Bundle B0, B1;
+    bundle_load<UPPER>(B0, S, rp, slot, 0, lane);
+    for (;;) {
+        // ---- locate and prefetch record t+1
+        int ni = i, nr = r + 1, nslot = slot, nnrec = nrec;
+        const uint8_t* nrp = rp + *(const uint16_t*)(rp + 6);
+        bool has_next = true;
+        while (nr >= nnrec) {
+            if (ni + 1 >= ie) { has_next = false; break; }
+            ++ni;
+            const unsigned q = q0 + ni;
+            nslot = q % SPCG_NCHUNK;
+            mbar_wait(&S.vfull[nslot], (q / SPCG_NCHUNK) & 1, P.sc);
+            if (aborted(P.sc)) { *rz_io = rz; return; }
+            const uint8_t* ch = S.chunks + (size_t)nslot * SPCG_CHUNK_BYTES;
+            nnrec = *(const uint16_t*)ch;
+            nrp = ch + 16;
+            nr = 0;
+            if (nnrec == 0) {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&S.empty[nslot]);
+            }
+        }
+        if (has_next) bundle_load<UPPER>(B1, S, nrp, nslot, nr, lane);
+        if (lane == 0) S.progress[0] = recn;
+        if (lane == 0) hbeat(P, 4, ((unsigned long long)(i + 1) << 40) | (unsigned long long)recn);
+        // ---- compute record t
+        const int fl = B0.fl;
+        double acc;
+        if ((fl & (REC_FIRST | REC_LAST | REC_EXT | REC_WIDE)) == (REC_FIRST | REC_LAST)) {
+            // fast path: one record per row, <= WP ring entries, no cross-CTA dependency
+            double d[WP];
+#pragma unroll
+            for (int k = 0; k < WP; ++k) d[k] = S.yring[B0.sidx[k]];
+            acc = B0.vec;
+#pragma unroll
+            for (int k = 0; k < WP; ++k) acc = fma(-B0.v[k], d[k], acc);   // v = 0 off-entry
+        } else {
+            const int len = meta_len(B0.meta), ne = meta_ne(B0.meta);
+            const Rec R(B0.p);
+            if (fl & REC_FIRST) {
+                double e = 0.0;
+                if (ne > 0) {
+                    const unsigned m = *(volatile unsigned*)side_mask(S, B0.slot, B0.r);
+                    if (m & (1u << lane)) { __threadfence_block(); e = side_ext(S, B0.slot, B0.r)[lane]; }
+                    else e = ext_wait(R, lane, ne, mb, ep, P.sc);
+                }
+                acc = B0.vec - e;
+            } else {
+                acc = acc_carry;
+                for (int k = 0; k < ne; ++k)
+                    acc = fma(-R.val(k, lane), ll_wait(mb + (-R.src(k, lane) - 1), ep, P.sc), acc);
+            }
+            if (!(fl & REC_WIDE)) {
+                double d[WP];
+#pragma unroll
+                for (int k = 0; k < WP; ++k) d[k] = S.yring[B0.sidx[k]];
+#pragma unroll
+                for (int k = 0; k < WP; ++k) acc = fma(-B0.v[k], d[k], acc);
+            } else {
+                acc = ring_terms_dispatch(R.w(), B0.p, lane, ne, len, S.yring, acc);
+            }
+        }
+        if (fl & REC_LAST) {
+            const bool live = B0.row >= 0;
+            if (UPPER) {
+                acc *= B0.dinv;
+                const double ri = (fl & REC_FIRST) ? B0.aux : ((rdot && live) ? __ldcg(rdot + B0.row) : 0.0);
+                if (live) rz = fma(ri, acc, rz);
+                if (PRO && live) P.p[B0.row] = acc;
+            }
+            if (live) {
+                S.yring[(B0.row - pb) & mask] = acc;
+                out[B0.row] = acc;
+                if (meta_pub(B0.meta)) ll_store((uint4*)mb + B0.row, acc, ep);
+            }
+        }
+        acc_carry = acc;
+        __syncwarp();
+        if (!has_next || ni != i) {                  // leaving this record's chunk
+            if (lane == 0) mbar_arrive(&S.empty[slot]);
+        }
+        if (!has_next || aborted(P.sc)) break;
+        i = ni; r = nr; slot = nslot; nrec = nnrec; rp = nrp;
+        ++recn;
+        B0 = B1;
+    }
+    *rz_io = rz;
+}
+
+// One triangular-solve phase of a part: chunks [c0, c1) of its stream (L section,
+// U section or both).  All threads of the CTA call it.
+__device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st, int c0, int c1, int cu, int kind,
+                              const double* rin, double* y, const double* yin, double* z, const double* rdot,
+                              unsigned ep, double alpha, double& rr, double& rz, int64_t pb) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int mask = P.ring - 1;
+    const unsigned q0 = st.q;
+    const long long rec0 = st.rec;
+    const int nch = c1 - c0;
+    if (warp == PRODUCER_WARP) {
+        // chunk sizes are read 32 at a time by the whole warp (one round trip), then
+        // lane 0 issues the bulk copies as ring slots free up
+        for (int b0 = 0; b0 < nch; b0 += 32) {
+            const int cnt = min(32, nch - b0);
+            unsigned my_bytes = 0;
+            if (lane < cnt) my_bytes = __ldg(P.chunk_bytes + c0 + b0 + lane);
+            for (int t = 0; t < cnt; ++t) {
+                if (aborted(P.sc)) break;                                // warp-uniform
+                const unsigned bytes = __shfl_sync(0xffffffffu, my_bytes, t);
+                if (lane == 0) {
+                    const unsigned q = q0 + b0 + t, slot = q % SPCG_NCHUNK, use = q / SPCG_NCHUNK;
+                    mbar_wait(&S.empty[slot], (use & 1) ^ 1, P.sc);
+                    hbeat(P, 0, ((unsigned long long)(st.k + 1) << 40) | q);
+                    mbar_arrive_tx(&S.full[slot], bytes);
+                    bulk_g2s(S.chunks + (size_t)slot * SPCG_CHUNK_BYTES,
+                             P.stream + (size_t)(c0 + b0 + t) * SPCG_CHUNK_BYTES, bytes, &S.full[slot]);
+                }
+                __syncwarp();
+            }
+        }
+    } else if (warp >= VEC_WARP0 && warp < SOLVER_WARP0) {
+        const int v = warp - VEC_WARP0;
+        bool waited_ldone = false;
+        long long recn = rec0;
+        for (int i = 0; i < nch; ++i) {
+            const unsigned q = q0 + i, slot = q % SPCG_NCHUNK, use = q / SPCG_NCHUNK;
+            if (c0 + i >= cu && !waited_ldone && cu > c0) {   // y of the L section must be complete
+                mbar_wait(S.ldone, st.ldone_uses & 1, P.sc);
+                waited_ldone = true;
+            }
+            if (v == 0 && lane == 0) hbeat(P, 1, ((unsigned long long)(st.k + 1) << 40) | q);
+            mbar_wait(&S.full[slot], use & 1, P.sc);
+            if (aborted(P.sc)) break;
+            const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
+            const int nrec = *(const uint16_t*)ch;
+            const uint8_t* rp = ch + 16;
+            // records are dealt to the vector warps by their global index (<= 1 per warp per chunk)
+            for (int r = 0; r < nrec; ++r, ++recn) {
+                Rec R(rp);
+                rp += R.bytes();
+                if ((int)(recn % NVEC) != v || !(R.flags() & REC_FIRST)) continue;
+                const int row = R.row(lane);
+                double* vec = side_vec(S, slot, r);
+                if (row >= 0) {
+                    if (!(R.flags() & REC_UPPER)) {
+                        double ri;
+                        if (kind == K_ITER) {                  // all four loads before any store
+                            const double r0 = P.r[row], w0 = P.w[row], x0 = P.x[row], p0 = P.p[row];
+                            ri = r0 - alpha * w0;
+                            P.r[row] = ri;
+                            P.x[row] = x0 + alpha * p0;
+                        } else {
+                            ri = rin[row];
+                            if (kind == K_PRO) {
+                                if (rin != P.r) P.r[row] = ri;
+                                if (!P.use_x0) P.x[row] = 0.0;
+                            }
+                        }
+                        rr = fma(ri, ri, rr);
+                        vec[lane] = ri;
+                    } else {
+                        const double y0 = __ldcg(yin + row);
+                        const double a0 = rdot ? __ldcg(rdot + row) : 0.0;
+                        vec[lane] = y0;
+                        side_aux(S, slot, r)[lane] = a0;
+                    }
+                }
+                if (lane == 0) *side_mask(S, slot, r) = 0u;
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.vfull[slot]);
+        }
+    } else if (warp == POLLER_WARP) {
+        long long recn = rec0;
+        for (int i = 0; i < nch; ++i) {
+            const unsigned q = q0 + i, slot = q % SPCG_NCHUNK, use = q / SPCG_NCHUNK;
+            if (lane == 0) hbeat(P, 2, ((unsigned long long)(st.k + 1) << 40) | q);
+            mbar_wait(&S.vfull[slot], use & 1, P.sc);
+            if (aborted(P.sc)) break;
+            const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
+            const int nrec = *(const uint16_t*)ch;
+            const uint8_t* rp = ch + 16;
+            for (int r = 0; r < nrec; ++r, ++recn) {
+                Rec R(rp);
+                rp += R.bytes();
+                if (lane == 0) hbeat(P, 3, ((unsigned long long)(st.k + 1) << 40) | (unsigned long long)recn);
+                if (!(R.flags() & REC_FIRST)) continue;
+                const int2 lw = R.lane(lane);
+                const int ne = lw.x >= 0 ? meta_ne((unsigned)lw.y) : 0;
+                if (!__any_sync(0xffffffffu, ne > 0)) continue;
+                const uint4* mb = (R.flags() & REC_UPPER) ? P.mbU : P.mbL;
+                bool need = ne > 0;
+                unsigned it = 0;
+                const long long tp0 = clock64();
+                for (;;) {                                     // warp-uniform control flow
+                    __syncwarp();
+                    const long long pmin = __shfl_sync(0xffffffffu, (long long)S.progress[0], 0);
+                    if (lane == 0) { hbeat(P, 6, (unsigned long long)pmin); hbeat(P, 7, it); }
+                    if (pmin >= recn) break;                   // the solver is here: it polls itself
+                    if (recn <= pmin + POLL_AHEAD) {           // close enough: values may be there
+                        double e = 0.0;
+                        const bool ok = need && ext_try(R, lane, ne, mb, ep, e);
+                        __syncwarp();
+                        if (ok) {
+                            side_ext(S, slot, r)[lane] = e;
+                            __threadfence_block();
+                            atomicOr(side_mask(S, slot, r), 1u << lane);
+                            need = false;
+                        }
+                        if (__ballot_sync(0xffffffffu, need) == 0u) break;
+                    } else {
+                        __nanosleep(64);
+                    }
+                    if ((++it & 255) == 0) {
+                        const bool late = __shfl_sync(0xffffffffu, clock64() - tp0 > SPIN_TIMEOUT_CYC, 0);
+                        if (late && lane == 0) atomicExch(&P.sc->abort, 1);
+                        if (late || aborted(P.sc)) break;
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.empty[slot]);
+        }
+    } else {
+        // ---------------- solver warp (one per CTA)
+        const int ncL = (c0 < cu) ? min(cu, c1) - c0 : 0;       // chunks of the L section
+        if (lane == 0) trace_mark(P, st.k, 8 + 4 * blockIdx.x + 0);
+        if (ncL > 0) {
+            double dummy = 0.0;
+            solver_section<false, false>(P, S, q0, 0, ncL, rec0, y, nullptr, P.mbL, ep, pb, mask, &dummy);
+            __syncwarp();
+            if (lane == 0 && c1 > cu) {
+                mbar_arrive(S.ldone);                              // y of the L section complete
+                trace_mark(P, st.k, 8 + 4 * blockIdx.x + 1);
+            }
+        }
+        if (ncL < nch) {
+            long long n = 0;                                        // U records continue the numbering
+            for (int t = 0; t < ncL; ++t) n += *(const uint16_t*)(P.stream + (size_t)(c0 + t) * SPCG_CHUNK_BYTES);
+            if (kind == K_PRO)
+                solver_section<true, true>(P, S, q0, ncL, nch, rec0 + n, z, rdot, P.mbU, ep, pb, mask, &rz);
+            else
+                solver_section<true, false>(P, S, q0, ncL, nch, rec0 + n, z, rdot, P.mbU, ep, pb, mask, &rz);
+        }
+        if (lane == 0) trace_mark(P, st.k, 8 + 4 * blockIdx.x + 2);
+    }
+    // all roles walked the same chunk sequence
+    st.q = q0 + nch;
+    if (cu > c0 && c1 > cu) st.ldone_uses++;
+    __syncthreads();
+    // records count for the next phase (every role counts the same)
+    if (threadIdx.x == 0) {
+        long long n = 0;
+        for (int i = 0; i < nch; ++i) n += *(const uint16_t*)(P.stream + (size_t)(c0 + i) * SPCG_CHUNK_BYTES);
+        S.progress[SPCG_NSOLVER] = rec0 + n;
+    }
+    __syncthreads();
+    st.rec = S.progress[SPCG_NSOLVER];
+    if (threadIdx.x == 0) trace_mark(P, st.k, 8 + 4 * blockIdx.x + 3);
+    if (threadIdx.x == 0)
+        for (int i = 0; i < SPCG_NSOLVER; ++i) S.progress[i] = st.rec - 1;
+    __syncthreads();
 }
 
 // M = I (K = -1): z = r with the fused update
@@ -377,26 +960,42 @@ __device__ void phase_pupdate(const Params& P, double beta) {
     for (int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x; i < P.n; i += stride) P.p[i] = fma(beta, P.p[i], P.z[i]);
 }
 
-// z = M^-1 r : forward then backward solve (or identity)
+// Triangular solves of Alg. 1 line 13.  sec: 1 = forward (L) only, 2 = backward
+// (U) only, 3 = both (z = U^-1 L^-1 r).  L reads rin, writes y; U reads yin, writes z.
 template <int STRAT>
-__device__ void precond(const Params& P, int kind, const double* rin, double* y, double* z, const double* rdot,
-                        unsigned ep, double alpha, double& rr, double& rz, double* ring, unsigned& gen) {
+__device__ void tri_solve(const Params& P, int sec, int kind, const double* rin, double* y, const double* yin,
+                          double* z, const double* rdot, unsigned ep, double alpha, double& rr, double& rz,
+                          double* dyn, unsigned& gen, const ChunkSmem& CS, PipeState& ps) {
     if (P.identity) {
-        phase_identity(P, kind, rin, z, rdot, alpha, rr, rz);
+        if (sec == 2) phase_identity(P, K_APPLY, yin, z, rdot, 0.0, rr, rz);
+        else phase_identity(P, kind, rin, sec == 1 ? y : z, sec == 3 ? rdot : nullptr, alpha, rr, rz);
         return;
     }
-    tri_phase<STRAT, false>(P, P.L, kind, rin, y, nullptr, P.mbL, ep, alpha, rr, ring, gen);
-    if (STRAT == ST_SYNCFREE) grid_sync(P.sc, gen);   // r_i / y_i written by another warp
-    tri_phase<STRAT, true>(P, P.U, kind, y, z, rdot, P.mbU, ep, 0.0, rz, ring, gen);
+    if (STRAT == ST_CHUNKED) {
+        const int c = blockIdx.x;
+        const int cb = P.part_chunk[c], cu = P.part_uchunk[c], ce = P.part_chunk[c + 1];
+        const int c0 = (sec & 1) ? cb : cu, c1 = (sec & 2) ? ce : cu;
+        chunked_phase(P, CS, ps, c0, c1, cu, kind, rin, y, yin, z, rdot, ep, alpha, rr, rz, P.part_begin[c]);
+        return;
+    }
+    if (sec & 1) tri_phase<STRAT, false>(P, P.L, kind, rin, y, nullptr, P.mbL, ep, alpha, rr, dyn, gen);
+    if (STRAT == ST_SYNCFREE && sec == 3) grid_sync(P.sc, gen);   // r_i / y_i written by another warp
+    if (sec & 2) tri_phase<STRAT, true>(P, P.U, kind, yin, z, rdot, P.mbU, ep, 0.0, rz, dyn, gen);
 }
 
 template <int STRAT>
 __global__ void __launch_bounds__(BLOCK, 1) spcg_pcg_kernel(Params P) {
-    extern __shared__ double ring[];
+    extern __shared__ __align__(128) double dyn[];
+    double* ring = dyn;
     unsigned gen = 0;
     if (threadIdx.x == 0) gen = ld_acquire_u32(&P.sc->bar_gen);
-    if (STRAT == ST_CHUNKED)
+    ChunkSmem CS{};
+    PipeState ps{0u, 0u, 0ll, -1ll};
+    if (STRAT == ST_CHUNKED) {
+        CS = chunk_smem(dyn, P.ring);
         for (int i = threadIdx.x; i < P.ring; i += BLOCK) ring[i] = 0.0;
+        chunk_init(CS);
+    }
     __syncthreads();
     unsigned app = 0;
 
@@ -405,13 +1004,11 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_pcg_kernel(Params P) {
         if (P.mode == M_SPMV) {
             phase_spmv(P, P.in, P.out, a);
         } else if (P.mode == M_LOWER) {
-            if (P.identity) phase_identity(P, K_APPLY, P.in, P.out, nullptr, 0.0, a, b);
-            else tri_phase<STRAT, false>(P, P.L, K_APPLY, P.in, P.out, nullptr, P.mbL, P.epoch, 0.0, a, ring, gen);
+            tri_solve<STRAT>(P, 1, K_APPLY, P.in, P.out, nullptr, nullptr, nullptr, P.epoch, 0.0, a, b, ring, gen, CS, ps);
         } else if (P.mode == M_UPPER) {
-            if (P.identity) phase_identity(P, K_APPLY, P.in, P.out, P.aux, 0.0, a, b);
-            else tri_phase<STRAT, true>(P, P.U, K_APPLY, P.in, P.out, P.aux, P.mbU, P.epoch, 0.0, b, ring, gen);
+            tri_solve<STRAT>(P, 2, K_APPLY, nullptr, nullptr, P.in, P.out, P.aux, P.epoch, 0.0, a, b, ring, gen, CS, ps);
         } else {
-            precond<STRAT>(P, K_APPLY, P.in, P.y, P.out, P.aux, P.epoch, 0.0, a, b, ring, gen);
+            tri_solve<STRAT>(P, 3, K_APPLY, P.in, P.y, P.y, P.out, P.aux, P.epoch, 0.0, a, b, ring, gen, CS, ps);
         }
         block_partials(a, b, P.partials, 0, 1);
         grid_sync(P.sc, gen);
@@ -437,7 +1034,7 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_pcg_kernel(Params P) {
         r_src = P.r;
     }
     double rr_l = 0.0, rz_l = 0.0;
-    precond<STRAT>(P, K_PRO, r_src, P.y, P.z, P.r, P.epoch + app, 0.0, rr_l, rz_l, ring, gen);
+    tri_solve<STRAT>(P, 3, K_PRO, r_src, P.y, P.y, P.z, P.r, P.epoch + app, 0.0, rr_l, rz_l, ring, gen, CS, ps);
     ++app;
     block_partials(rz_l, rr_l, P.partials, 0, 1);
     grid_sync(P.sc, gen);
@@ -451,7 +1048,10 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_pcg_kernel(Params P) {
         if (blockIdx.x == 0 && threadIdx.x == 0 && P.rhist && k < P.rhist_cap) P.rhist[k] = rn;
         if (rn < P.eps || rr == 0.0) { status = SPCG_OK; break; }                       // lines 6-7
         if (k == P.kmax) { status = P.eps > 0.0 ? SPCG_NOT_CONVERGED : SPCG_OK; break; }  // A14
-        if (ld_volatile_int(&P.sc->abort)) { status = SPCG_ERR_INTERNAL; break; }
+        if (__syncthreads_or(ld_volatile_int(&P.sc->abort))) { status = SPCG_ERR_INTERNAL; break; }   // CTA-uniform
+        ps.k = k;
+        if (threadIdx.x == 0) hbeat(P, 5, (unsigned long long)k);
+        if (blockIdx.x == 0 && threadIdx.x == 0) trace_mark(P, k, 0);
         // line 9-10: w = A p, sigma = (p, w), alpha = rho / sigma
         double pw = 0.0;
         phase_spmv(P, P.p, P.w, pw);
@@ -461,13 +1061,16 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_pcg_kernel(Params P) {
         global_sums(P.partials, 2, -1, sigma, unused);
         if (!(sigma > 0.0) || !isfinite(sigma) || !isfinite(rho)) { status = SPCG_ERR_BREAKDOWN; break; }
         const double alpha = rho / sigma;
+        if (blockIdx.x == 0 && threadIdx.x == 0) trace_mark(P, k, 1);
         // lines 11-13 (+ ||r||^2, (r, z))
         rr_l = 0.0;
         rz_l = 0.0;
-        precond<STRAT>(P, K_ITER, P.r, P.y, P.z, P.r, P.epoch + app, alpha, rr_l, rz_l, ring, gen);
+        tri_solve<STRAT>(P, 3, K_ITER, P.r, P.y, P.y, P.z, P.r, P.epoch + app, alpha, rr_l, rz_l, ring, gen, CS, ps);
         ++app;
+        if (blockIdx.x == 0 && threadIdx.x == 0) trace_mark(P, k, 2);
         block_partials(rz_l, rr_l, P.partials, 0, 1);
         grid_sync(P.sc, gen);
+        if (blockIdx.x == 0 && threadIdx.x == 0) trace_mark(P, k, 3);
         double rho_new;
         global_sums(P.partials, 0, 1, rho_new, rr);
         // lines 14-15
@@ -475,6 +1078,7 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_pcg_kernel(Params P) {
         rho = rho_new;
         phase_pupdate(P, beta);
         grid_sync(P.sc, gen);
+        if (blockIdx.x == 0 && threadIdx.x == 0) trace_mark(P, k, 4);
         ++k;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -508,7 +1112,18 @@ struct spcg_device_s {
     int64_t bytes = 0;
     unsigned epoch = 1;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    unsigned long long* trace = nullptr;
+    unsigned long long* hb = nullptr;
 };
+
+// debug: copy the heartbeat array while a kernel may still be running (own non-blocking stream)
+extern "C" int spcg_dbg_heartbeats(void* handle_dev, unsigned long long* out, int n) {
+    spcg_device_t* d = (spcg_device_t*)handle_dev;
+    if (!d || !d->hb) return -1;
+    int m = std::min(n, 8 * d->parts);
+    for (int i = 0; i < m; ++i) out[i] = ((volatile unsigned long long*)d->hb)[i];
+    return m;
+}
 
 template <class T>
 static spcg_status_t upload(spcg_device_t* d, const std::vector<T>& v, const T** out) {
@@ -591,6 +1206,10 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
     UP(lay.A.val, P.A.val);
     if (upload_tri(d, lay.L, P.L) || upload_tri(d, lay.U, P.U)) { spcg_dev_destroy(d); return SPCG_ERR_CUDA; }
     UP(lay.part_begin, P.part_begin);
+    UP(lay.S.bytes, P.stream);
+    UP(lay.S.part_chunk, P.part_chunk);
+    UP(lay.S.part_uchunk, P.part_uchunk);
+    UP(lay.S.chunk_bytes, P.chunk_bytes);
     void* p;
     const size_t vb = (size_t)n * sizeof(double);
 #define AL(bytes_, dst, T)                                                  \
@@ -614,10 +1233,11 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         spcg_dev_destroy(d);
         return SPCG_ERR_CUDA;
     }
-    d->smem = lay.strategy == ST_CHUNKED ? (size_t)lay.ring * sizeof(double) : 0;
+    d->smem = lay.strategy == ST_CHUNKED ? chunked_smem_bytes(lay.ring) : 0;
     void* kfn = pick_kernel(d->strategy);
     // one attribute value for every handle: the largest ring any layout builds (16384 entries)
-    if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, 16384 * (int)sizeof(double)) != cudaSuccess) {
+    const int smem_max = lay.strategy == ST_CHUNKED ? (int)chunked_smem_bytes(16384) : 0;
+    if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max) != cudaSuccess) {
         spcg::set_error("cannot reserve shared memory for the ring");
         spcg_dev_destroy(d);
         return SPCG_ERR_CUDA;
@@ -629,6 +1249,21 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         spcg::set_error("persistent grid does not fit co-resident");
         spcg_dev_destroy(d);
         return SPCG_ERR_CUDA;
+    }
+    if (getenv("SPCG_TRACE")) {
+        void* hp = nullptr;
+        if (cudaHostAlloc(&hp, sizeof(unsigned long long) * 8 * (size_t)lay.parts, cudaHostAllocMapped) == cudaSuccess) {
+            memset(hp, 0, sizeof(unsigned long long) * 8 * (size_t)lay.parts);
+            d->hb = (unsigned long long*)hp;                 // host view (zero-copy, readable any time)
+            void* dp = nullptr;
+            cudaHostGetDevicePointer(&dp, hp, 0);
+            P.hb = (unsigned long long*)dp;
+        }
+        void* tp = nullptr;
+        if (alloc(d, sizeof(unsigned long long) * (8 + 4 * (size_t)lay.parts + 400), &tp) == SPCG_OK) {
+            d->trace = (unsigned long long*)tp;
+            P.trace = d->trace;
+        }
     }
     if (cudaEventCreate(&d->ev0) != cudaSuccess || cudaEventCreate(&d->ev1) != cudaSuccess) {
         spcg_dev_destroy(d);
@@ -686,6 +1321,7 @@ spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, doubl
     CK(cudaMallocAsync((void**)&dh, sizeof(double) * cap, d->stream));
     P.rhist = dh;
     P.rhist_cap = cap;
+    if (d->trace) CK(cudaMemsetAsync(d->trace, 0, sizeof(unsigned long long) * (8 + 4 * (size_t)d->parts + 400), d->stream));
     CK(cudaEventRecord(d->ev0, d->stream));
     spcg_status_t st = launch(d, P);
     if (st != SPCG_OK) { cudaFreeAsync(dh, d->stream); return st; }
@@ -708,6 +1344,16 @@ spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, doubl
     info->converged = (sc.status == SPCG_OK && eps > 0.0) ? 1 : 0;
     info->iter_phase_ms = ms;
     if (sc.status == SPCG_ERR_INTERNAL) report_abort(d, sc);
+    if (d->trace) {
+        std::vector<unsigned long long> t(8 + 4 * (size_t)d->parts + 400);
+        cudaMemcpy(t.data(), d->trace, t.size() * 8, cudaMemcpyDeviceToHost);
+        if (FILE* f = fopen(getenv("SPCG_TRACE"), "a")) {
+            fprintf(f, "trace parts=%d", d->parts);
+            for (auto v : t) fprintf(f, " %llu", v);
+            fprintf(f, "\n");
+            fclose(f);
+        }
+    }
     return sc.status;
 }
 
