@@ -88,6 +88,7 @@ constexpr int SPCG_MAXREC = 8;          // records per chunk (side-data slots)
 constexpr int SPCG_WCAP = 8;            // entry columns per record
 constexpr int SPCG_NSOLVER = 1;         // solver warps per CTA (one software-pipelined chain)
 constexpr int SPCG_REC_HDR = 272;       // 16 B header + 32 x {int32 row, uint32 meta}
+constexpr int SPCG_CHUNK_HDR = 32;      // u16 nrec, u16 -, u32 used, u16 rec_off[8], pad
 enum { REC_FIRST = 1, REC_LAST = 2, REC_SYNC = 4, REC_UPPER = 8, REC_EXT = 16, REC_WIDE = 32 };
 constexpr int SPCG_WP = 4;              // entry columns the pipelined solver keeps in registers
 
@@ -104,7 +105,8 @@ struct Layouts {
     int32_t strategy = SPCG_SPTRSV_LEVEL;
     int32_t parts = 1;
     int32_t ring = 0;              // entries of the shared-memory ring (chunked)
-    std::vector<int64_t> part_begin; // [parts+1] contiguous row ranges (chunked)
+    std::vector<int64_t> part_begin; // [parts+1] prefix of part sizes (chunked)
+    std::string partition;           // partition the inspector chose (chunked)
     SpmvLayout A;
     TriLayout L, U;
     ChunkStream S;                 // chunked executor only

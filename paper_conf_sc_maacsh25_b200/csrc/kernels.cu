@@ -37,7 +37,7 @@ using namespace spcg;
 
 namespace {
 
-constexpr int BLOCK = 384;
+constexpr int BLOCK = 256;
 constexpr int NWARP = BLOCK / 32;
 constexpr long long SPIN_TIMEOUT_CYC = 8ll * 1000 * 1000 * 1000;            // ~4 s of SM cycles: abort, never hang
 
@@ -379,16 +379,17 @@ __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const doub
 // Warp roles inside a CTA during a triangular-solve phase:
 //   warp 0        producer: one lane streams the part's record chunks into the
 //                 shared-memory ring with cp.async.bulk (TMA), mbarrier complete_tx
-//   warp 1        poller: a few records ahead of the solvers, polls the ready flags
+//   warps 1..2    pollers: a few records ahead of the solver, poll the ready flags
 //                 of cross-CTA dependencies and leaves their partial sum in smem
-//   warps 2..10   vector warps: per record, the dynamic per-row operands (fused
+//   warps 3..6    vector warps: per record, the dynamic per-row operands (fused
 //                 x/r update and ||r||^2 for L; y_i and r_i for U)
-//   warp 11       solver warp: the dependency chain, software-pipelined one record
+//   warp 7        solver warp: the dependency chain, software-pipelined one record
 //                 ahead so only ring gather -> FMA -> store sits on the critical path
 constexpr int PRODUCER_WARP = 0;
 constexpr int POLLER_WARP = 1;
-constexpr int VEC_WARP0 = 2;
-constexpr int NVEC = 9;
+constexpr int NPOLL = 2;                          // poller warps (records alternate)
+constexpr int VEC_WARP0 = POLLER_WARP + NPOLL;
+constexpr int NVEC = 4;
 constexpr int SOLVER_WARP0 = VEC_WARP0 + NVEC;
 static_assert(SOLVER_WARP0 + SPCG_NSOLVER == NWARP, "warp roles must fill the CTA");
 constexpr int POLL_AHEAD = 8;                     // records
@@ -439,19 +440,23 @@ __device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
         : "memory");
     return ok != 0;
 }
-__device__ __noinline__ void mbar_wait_slow(uint64_t* b, unsigned parity, Scal* sc) {
+// returns false if the wait was abandoned because of an abort (callers make
+// that warp-uniform before acting on it)
+__device__ __noinline__ bool mbar_wait_slow(uint64_t* b, unsigned parity, Scal* sc) {
     const long long t0 = clock64();
     unsigned it = 0;
     while (!mbar_try(b, parity)) {
         if ((++it & 3) == 0) {
-            if (ld_volatile_int(&sc->abort)) return;
-            if (clock64() - t0 > SPIN_TIMEOUT_CYC) { atomicExch(&sc->abort, 1); return; }
+            if (ld_volatile_int(&sc->abort)) return false;
+            if (clock64() - t0 > SPIN_TIMEOUT_CYC) { atomicExch(&sc->abort, 1); return false; }
         }
     }
+    return true;
 }
-__device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity, Scal* sc) {
-    if (!mbar_try(b, parity)) mbar_wait_slow(b, parity, sc);
+__device__ __forceinline__ bool mbar_wait(uint64_t* b, unsigned parity, Scal* sc) {
+    return mbar_try(b, parity) || mbar_wait_slow(b, parity, sc);
 }
+__device__ __forceinline__ bool warp_ok(bool ok) { return __all_sync(0xffffffffu, ok); }
 // After an abort the ring may hold stale chunks: roles must stop parsing them.
 // Warp-collective code must take this decision warp-uniformly (a per-lane read
 // of a racy flag lets lanes disagree; a divergent break then deadlocks the
@@ -486,7 +491,7 @@ __device__ void chunk_init(const ChunkSmem& S) {
         for (int i = 0; i < SPCG_NCHUNK; ++i) {
             mbar_init(&S.full[i], 1);
             mbar_init(&S.vfull[i], NVEC);
-            mbar_init(&S.empty[i], SPCG_NSOLVER + 1);
+            mbar_init(&S.empty[i], SPCG_NSOLVER + NPOLL);
         }
         mbar_init(S.ldone, SPCG_NSOLVER);
         for (int i = 0; i < SPCG_NSOLVER; ++i) S.progress[i] = -1;
@@ -599,160 +604,199 @@ __device__ __forceinline__ double ring_terms_dispatch(int wd, const uint8_t* p, 
     }
 }
 
-// One record's operands as held in registers by the pipelined solver warp.
+// ---- solver warp ------------------------------------------------------------
+// A record's operands, loaded ahead of its computation (see solver_section).
 constexpr int WP = SPCG_WP;
-struct Bundle {
+struct Prep {
     const uint8_t* p;
-    int fl, slot, r, row;
+    int fl, wd, row, r;
     unsigned meta;
-    double vec, dinv, aux;
     int sidx[WP];
     double v[WP];
+    double vec, dinv, aux;
+};
+
+struct SolveCtx {          // per-section constants of the solver warp
+    double* yring;
+    const ChunkSmem* S;
+    double* out;
+    const double* rdot;
+    double* pvec;          // p (prologue: p0 = z0)
+    const uint4* mb;
+    Scal* sc;
+    unsigned ep;
+    int64_t pb;
+    int mask;
 };
 
 template <bool UPPER>
-__device__ __forceinline__ void bundle_load(Bundle& B, const ChunkSmem& S, const uint8_t* p, int slot, int r, int lane) {
-    B.p = p;
-    B.slot = slot;
-    B.r = r;
-    const uint4 h = *(const uint4*)p;
-    B.fl = (int)(h.x >> 16);
-    const int wd = (int)(h.x & 0xffffu);
-    const int2 lw = *(const int2*)(p + 16 + 8 * lane);
-    B.row = lw.x;
-    B.meta = (unsigned)lw.y;
-    const int len = meta_len(B.meta), ne = meta_ne(B.meta);
-    const uint8_t* sp = p + SPCG_REC_HDR + 4 * lane;
-    const uint8_t* vp = p + SPCG_REC_HDR + 128 * wd + 8 * lane;
+__device__ __forceinline__ void prep_record(Prep& X, const ChunkSmem& S, const uint8_t* ch, int slot, int r, int lane) {
+    X.r = r;
+    X.p = ch + *(const uint16_t*)(ch + 8 + 2 * r);
+    const uint4 h = *(const uint4*)X.p;
+    X.fl = (int)(h.x >> 16);
+    X.wd = (int)(h.x & 0xffffu);
+    const int2 lw = *(const int2*)(X.p + 16 + 8 * lane);
+    X.row = lw.x;
+    X.meta = (unsigned)lw.y;
+    const int len = meta_len(X.meta), ne = meta_ne(X.meta);
+    const uint8_t* sp = X.p + SPCG_REC_HDR + 4 * lane;
+    const uint8_t* vp = X.p + SPCG_REC_HDR + 128 * X.wd + 8 * lane;
 #pragma unroll
     for (int k = 0; k < WP; ++k) {
-        const bool on = k >= ne && k < len && k < wd;      // ring entries only
-        B.sidx[k] = on ? *(const int*)(sp + 128 * k) : 0;
-        B.v[k] = on ? *(const double*)(vp + 256 * k) : 0.0;
+        const bool on = k >= ne && k < len && k < X.wd;     // ring entries in registers
+        X.sidx[k] = on ? *(const int*)(sp + 128 * k) : 0;
+        X.v[k] = on ? *(const double*)(vp + 256 * k) : 0.0;
     }
-    B.vec = side_vec(S, slot, r)[lane];                     // meaningful on FIRST records
+    X.vec = side_vec(S, slot, r)[lane];
     if (UPPER) {
-        B.dinv = (B.fl & REC_LAST) ? *(const double*)(p + SPCG_REC_HDR + 384 * wd + 8 * lane) : 1.0;
-        B.aux = side_aux(S, slot, r)[lane];
+        const bool fast_last = (X.fl & (REC_LAST | REC_WIDE)) == REC_LAST;
+        X.dinv = fast_last ? *(const double*)(X.p + SPCG_REC_HDR + 384 * X.wd + 8 * lane) : 1.0;
+        X.aux = side_aux(S, slot, r)[lane];
     }
 }
 
-// The solver warp over one section (all L records or all U records of the part),
-// software-pipelined one record deep: while record t computes, record t+1's
-// header, lane word, entries and side operands are already in registers, so
-// only ring gather -> FMA chain -> ring store is on the dependency path.
+// row epilogue (Alg. 1 line 13 output + (r,z) + publication)
 template <bool UPPER, bool PRO>
-__device__ __noinline__ void solver_section(const Params& P, const ChunkSmem& S, unsigned q0, int ib, int ie,
-                                            long long recn, double* out, const double* rdot, const uint4* mb,
-                                            unsigned ep, int64_t pb, int mask, double* rz_io) {
-    const int lane = threadIdx.x & 31;
-    double rz = *rz_io;
-    double acc_carry = 0.0;          // accumulator of a row continued in the next record
-    // open the first chunk that has records (empty chunks are released at once)
-    int i = ib, nrec = 0, slot = 0;
-    const uint8_t* rp = nullptr;
-    for (;;) {
-        const unsigned q = q0 + i;
-        slot = q % SPCG_NCHUNK;
-        mbar_wait(&S.vfull[slot], (q / SPCG_NCHUNK) & 1, P.sc);
-        if (aborted(P.sc)) { *rz_io = rz; return; }
-        const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
-        nrec = *(const uint16_t*)ch;
-        rp = ch + 16;
-        if (nrec > 0) break;
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&S.empty[slot]);
-        if (++i >= ie) { *rz_io = rz; return; }
-    }
-    int r = 0;
-    Bundle B0, B1;
-    bundle_load<UPPER>(B0, S, rp, slot, 0, lane);
-    for (;;) {
-        // ---- locate and prefetch record t+1
-        int ni = i, nr = r + 1, nslot = slot, nnrec = nrec;
-        const uint8_t* nrp = rp + *(const uint16_t*)(rp + 6);
-        bool has_next = true;
-        while (nr >= nnrec) {
-            if (ni + 1 >= ie) { has_next = false; break; }
-            ++ni;
-            const unsigned q = q0 + ni;
-            nslot = q % SPCG_NCHUNK;
-            mbar_wait(&S.vfull[nslot], (q / SPCG_NCHUNK) & 1, P.sc);
-            if (aborted(P.sc)) { *rz_io = rz; return; }
-            const uint8_t* ch = S.chunks + (size_t)nslot * SPCG_CHUNK_BYTES;
-            nnrec = *(const uint16_t*)ch;
-            nrp = ch + 16;
-            nr = 0;
-            if (nnrec == 0) {
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&S.empty[nslot]);
-            }
+__device__ __forceinline__ void finish_row(const SolveCtx& C, int row, unsigned meta, double acc, double dinv,
+                                           double ri, double& rz) {
+    if (row >= 0) {
+        if (UPPER) {
+            acc *= dinv;
+            rz = fma(ri, acc, rz);
+            if (PRO) C.pvec[row] = acc;
         }
-        if (has_next) bundle_load<UPPER>(B1, S, nrp, nslot, nr, lane);
-        if (lane == 0) S.progress[0] = recn;
-        if (lane == 0) hbeat(P, 4, ((unsigned long long)(i + 1) << 40) | (unsigned long long)recn);
-        // ---- compute record t
-        const int fl = B0.fl;
-        double acc;
-        if ((fl & (REC_FIRST | REC_LAST | REC_EXT | REC_WIDE)) == (REC_FIRST | REC_LAST)) {
-            // fast path: one record per row, <= WP ring entries, no cross-CTA dependency
+        C.yring[meta >> 17] = acc;                    // part-local ring slot
+        C.out[row] = acc;
+        if (meta_pub(meta)) ll_store((uint4*)C.mb + row, acc, C.ep);
+    }
+}
+
+// general record: continuation of a row over several records, > WP entries, or
+// cross-CTA dependencies the poller did not resolve (rare: kept out of line).
+// Takes scalars only and returns {acc, rz} so no caller variable is address-taken.
+template <bool UPPER, bool PRO>
+__device__ __noinline__ double2 slow_record(const uint8_t* p, int fl, int wd, int row, unsigned meta, int r,
+                                            double vec, double aux, double acc_carry, double rz, double* side_rec,
+                                            double* yring, double* out, const double* rdot, double* pvec,
+                                            const uint4* mb, Scal* sc, unsigned ep, int64_t pb, int mask) {
+    const int lane = threadIdx.x & 31;
+    const Rec R(p);
+    const int len = meta_len(meta), ne = meta_ne(meta);
+    double acc;
+    if (fl & REC_FIRST) {
+        double e = 0.0;
+        if (row >= 0 && ne > 0) {
+            const unsigned m = *(volatile unsigned*)(side_rec + 96);
+            if (m & (1u << lane)) { __threadfence_block(); e = side_rec[64 + lane]; }
+            else e = ext_wait(R, lane, ne, mb, ep, sc);
+        }
+        acc = vec - e;
+    } else {
+        acc = acc_carry;
+        if (row >= 0)
+            for (int k = 0; k < ne; ++k) acc = fma(-R.val(k, lane), ll_wait(mb + (-R.src(k, lane) - 1), ep, sc), acc);
+    }
+    if (row >= 0) acc = ring_terms_dispatch(wd, p, lane, ne, len, yring, acc);
+    if ((fl & REC_LAST) && row >= 0) {
+        double a = acc;
+        if (UPPER) {
+            a *= R.dinv(lane);
+            const double ri = (fl & REC_FIRST) ? aux : (rdot ? __ldcg(rdot + row) : 0.0);
+            rz = fma(ri, a, rz);
+            if (PRO) pvec[row] = a;
+        }
+        yring[meta >> 17] = a;
+        out[row] = a;
+        if (meta_pub(meta)) ll_store((uint4*)mb + row, a, ep);
+        acc = a;
+    }
+    return make_double2(acc, rz);
+}
+
+__device__ unsigned long long* g_dbg_counts = nullptr;   // debug: [0] fast, [1] ext-fast, [2] slow
+template <bool UPPER, bool PRO>
+__device__ __forceinline__ void solve_record(const SolveCtx& C, const Prep& X, int slot, int lane, double& acc_carry,
+                                             double& rz) {
+    if ((X.fl & (REC_FIRST | REC_WIDE | REC_EXT)) == REC_FIRST) {
+        // fast path: whole row in this record, <= WP ring entries, no cross-CTA term
+        double d[WP];
+#pragma unroll
+        for (int k = 0; k < WP; ++k) d[k] = C.yring[X.sidx[k]];
+        double acc = X.vec;
+#pragma unroll
+        for (int k = 0; k < WP; ++k) acc = fma(-X.v[k], d[k], acc);   // v = 0 off-entry
+        finish_row<UPPER, PRO>(C, X.row, X.meta, acc, X.dinv, X.aux, rz);
+        acc_carry = acc;
+    } else if ((X.fl & (REC_FIRST | REC_WIDE)) == REC_FIRST) {
+        // cross-CTA terms: normally pre-resolved by the poller into the side slot
+        const int ne = meta_ne(X.meta);
+        const unsigned m = *(volatile unsigned*)side_mask(*C.S, slot, X.r);
+        const bool have = ne == 0 || (m >> lane) & 1u;
+        const bool all_have = __all_sync(0xffffffffu, have);
+        if (g_dbg_counts && lane == 0) atomicAdd(g_dbg_counts + (all_have ? 1 : 2), 1ull);
+        if (all_have) {
+            double e = 0.0;
+            if (ne > 0) { __threadfence_block(); e = side_ext(*C.S, slot, X.r)[lane]; }
             double d[WP];
 #pragma unroll
-            for (int k = 0; k < WP; ++k) d[k] = S.yring[B0.sidx[k]];
-            acc = B0.vec;
+            for (int k = 0; k < WP; ++k) d[k] = C.yring[X.sidx[k]];
+            double acc = X.vec - e;
 #pragma unroll
-            for (int k = 0; k < WP; ++k) acc = fma(-B0.v[k], d[k], acc);   // v = 0 off-entry
+            for (int k = 0; k < WP; ++k) acc = fma(-X.v[k], d[k], acc);
+            finish_row<UPPER, PRO>(C, X.row, X.meta, acc, X.dinv, X.aux, rz);
+            acc_carry = acc;
         } else {
-            const int len = meta_len(B0.meta), ne = meta_ne(B0.meta);
-            const Rec R(B0.p);
-            if (fl & REC_FIRST) {
-                double e = 0.0;
-                if (ne > 0) {
-                    const unsigned m = *(volatile unsigned*)side_mask(S, B0.slot, B0.r);
-                    if (m & (1u << lane)) { __threadfence_block(); e = side_ext(S, B0.slot, B0.r)[lane]; }
-                    else e = ext_wait(R, lane, ne, mb, ep, P.sc);
-                }
-                acc = B0.vec - e;
-            } else {
-                acc = acc_carry;
-                for (int k = 0; k < ne; ++k)
-                    acc = fma(-R.val(k, lane), ll_wait(mb + (-R.src(k, lane) - 1), ep, P.sc), acc);
-            }
-            if (!(fl & REC_WIDE)) {
-                double d[WP];
-#pragma unroll
-                for (int k = 0; k < WP; ++k) d[k] = S.yring[B0.sidx[k]];
-#pragma unroll
-                for (int k = 0; k < WP; ++k) acc = fma(-B0.v[k], d[k], acc);
-            } else {
-                acc = ring_terms_dispatch(R.w(), B0.p, lane, ne, len, S.yring, acc);
-            }
+            const double2 o = slow_record<UPPER, PRO>(X.p, X.fl, X.wd, X.row, X.meta, X.r, X.vec, X.aux, acc_carry, rz,
+                                                      side_vec(*C.S, slot, X.r), C.yring, C.out, C.rdot, C.pvec, C.mb,
+                                                      C.sc, C.ep, C.pb, C.mask);
+            acc_carry = o.x;
+            rz = o.y;
         }
-        if (fl & REC_LAST) {
-            const bool live = B0.row >= 0;
-            if (UPPER) {
-                acc *= B0.dinv;
-                const double ri = (fl & REC_FIRST) ? B0.aux : ((rdot && live) ? __ldcg(rdot + B0.row) : 0.0);
-                if (live) rz = fma(ri, acc, rz);
-                if (PRO && live) P.p[B0.row] = acc;
-            }
-            if (live) {
-                S.yring[(B0.row - pb) & mask] = acc;
-                out[B0.row] = acc;
-                if (meta_pub(B0.meta)) ll_store((uint4*)mb + B0.row, acc, ep);
-            }
-        }
-        acc_carry = acc;
-        __syncwarp();
-        if (!has_next || ni != i) {                  // leaving this record's chunk
-            if (lane == 0) mbar_arrive(&S.empty[slot]);
-        }
-        if (!has_next || aborted(P.sc)) break;
-        i = ni; r = nr; slot = nslot; nrec = nnrec; rp = nrp;
-        ++recn;
-        B0 = B1;
+    } else {
+        const double2 o = slow_record<UPPER, PRO>(X.p, X.fl, X.wd, X.row, X.meta, X.r, X.vec, X.aux, acc_carry, rz,
+                                                  side_vec(*C.S, slot, X.r), C.yring, C.out, C.rdot, C.pvec, C.mb,
+                                                  C.sc, C.ep, C.pb, C.mask);
+        acc_carry = o.x;
+        rz = o.y;
     }
-    *rz_io = rz;
+    __syncwarp();
+}
+
+// The solver warp over one section (all L or all U records of the part): per
+// chunk, records are fully unrolled with a ping-pong prefetch so that record
+// t+1's operands are in registers while record t computes; only ring gather ->
+// FMA chain -> ring store remains on the dependency path.
+template <bool UPPER, bool PRO>
+__device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSmem& S, unsigned q0, int ib, int ie,
+                                               long long recn, double& rz, const Params& P, long long kk) {
+    const int lane = threadIdx.x & 31;
+    double acc_carry = 0.0;
+    for (int i = ib; i < ie; ++i) {
+        const unsigned q = q0 + i;
+        const int slot = q % SPCG_NCHUNK;
+        if (!warp_ok(mbar_wait(&S.vfull[slot], (q / SPCG_NCHUNK) & 1, C.sc))) return;
+        const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
+        const int nrec = *(const uint16_t*)ch;
+        Prep A, B;
+        if (nrec > 0) prep_record<UPPER>(A, S, ch, slot, 0, lane);
+#pragma unroll
+        for (int r = 0; r < SPCG_MAXREC; r += 2) {
+            if (r + 1 < nrec) prep_record<UPPER>(B, S, ch, slot, r + 1, lane);
+            if (r < nrec) {
+                if (lane == 0) S.progress[0] = recn + r;
+                solve_record<UPPER, PRO>(C, A, slot, lane, acc_carry, rz);
+            }
+            if (r + 2 < nrec) prep_record<UPPER>(A, S, ch, slot, r + 2, lane);
+            if (r + 1 < nrec) {
+                if (lane == 0) S.progress[0] = recn + r + 1;
+                solve_record<UPPER, PRO>(C, B, slot, lane, acc_carry, rz);
+            }
+        }
+        recn += nrec;
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&S.empty[slot]);
+    }
 }
 
 // One triangular-solve phase of a part: chunks [c0, c1) of its stream (L section,
@@ -772,19 +816,22 @@ __device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st
             const int cnt = min(32, nch - b0);
             unsigned my_bytes = 0;
             if (lane < cnt) my_bytes = __ldg(P.chunk_bytes + c0 + b0 + lane);
-            for (int t = 0; t < cnt; ++t) {
-                if (aborted(P.sc)) break;                                // warp-uniform
+            bool ok = true;
+            for (int t = 0; t < cnt && ok; ++t) {
                 const unsigned bytes = __shfl_sync(0xffffffffu, my_bytes, t);
                 if (lane == 0) {
                     const unsigned q = q0 + b0 + t, slot = q % SPCG_NCHUNK, use = q / SPCG_NCHUNK;
-                    mbar_wait(&S.empty[slot], (use & 1) ^ 1, P.sc);
+                    ok = mbar_wait(&S.empty[slot], (use & 1) ^ 1, P.sc);
+                    if (ok) {
                     hbeat(P, 0, ((unsigned long long)(st.k + 1) << 40) | q);
                     mbar_arrive_tx(&S.full[slot], bytes);
                     bulk_g2s(S.chunks + (size_t)slot * SPCG_CHUNK_BYTES,
                              P.stream + (size_t)(c0 + b0 + t) * SPCG_CHUNK_BYTES, bytes, &S.full[slot]);
+                    }
                 }
-                __syncwarp();
+                ok = __shfl_sync(0xffffffffu, ok, 0);
             }
+            if (!ok) break;
         }
     } else if (warp >= VEC_WARP0 && warp < SOLVER_WARP0) {
         const int v = warp - VEC_WARP0;
@@ -793,20 +840,18 @@ __device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st
         for (int i = 0; i < nch; ++i) {
             const unsigned q = q0 + i, slot = q % SPCG_NCHUNK, use = q / SPCG_NCHUNK;
             if (c0 + i >= cu && !waited_ldone && cu > c0) {   // y of the L section must be complete
-                mbar_wait(S.ldone, st.ldone_uses & 1, P.sc);
+                if (!warp_ok(mbar_wait(S.ldone, st.ldone_uses & 1, P.sc))) break;
                 waited_ldone = true;
             }
             if (v == 0 && lane == 0) hbeat(P, 1, ((unsigned long long)(st.k + 1) << 40) | q);
-            mbar_wait(&S.full[slot], use & 1, P.sc);
-            if (aborted(P.sc)) break;
+            if (!warp_ok(mbar_wait(&S.full[slot], use & 1, P.sc))) break;
             const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
             const int nrec = *(const uint16_t*)ch;
-            const uint8_t* rp = ch + 16;
             // records are dealt to the vector warps by their global index (<= 1 per warp per chunk)
             for (int r = 0; r < nrec; ++r, ++recn) {
-                Rec R(rp);
-                rp += R.bytes();
-                if ((int)(recn % NVEC) != v || !(R.flags() & REC_FIRST)) continue;
+                if ((int)(recn % NVEC) != v) continue;
+                const Rec R(ch + *(const uint16_t*)(ch + 8 + 2 * r));
+                if (!(R.flags() & REC_FIRST)) continue;
                 const int row = R.row(lane);
                 double* vec = side_vec(S, slot, r);
                 if (row >= 0) {
@@ -838,21 +883,19 @@ __device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st
             __syncwarp();
             if (lane == 0) mbar_arrive(&S.vfull[slot]);
         }
-    } else if (warp == POLLER_WARP) {
+    } else if (warp >= POLLER_WARP && warp < POLLER_WARP + NPOLL) {
+        const int pw = warp - POLLER_WARP;
         long long recn = rec0;
         for (int i = 0; i < nch; ++i) {
             const unsigned q = q0 + i, slot = q % SPCG_NCHUNK, use = q / SPCG_NCHUNK;
-            if (lane == 0) hbeat(P, 2, ((unsigned long long)(st.k + 1) << 40) | q);
-            mbar_wait(&S.vfull[slot], use & 1, P.sc);
-            if (aborted(P.sc)) break;
+            if (lane == 0 && pw == 0) hbeat(P, 2, ((unsigned long long)(st.k + 1) << 40) | q);
+            if (!warp_ok(mbar_wait(&S.vfull[slot], use & 1, P.sc))) break;
             const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
             const int nrec = *(const uint16_t*)ch;
-            const uint8_t* rp = ch + 16;
             for (int r = 0; r < nrec; ++r, ++recn) {
-                Rec R(rp);
-                rp += R.bytes();
-                if (lane == 0) hbeat(P, 3, ((unsigned long long)(st.k + 1) << 40) | (unsigned long long)recn);
-                if (!(R.flags() & REC_FIRST)) continue;
+                const Rec R(ch + *(const uint16_t*)(ch + 8 + 2 * r));
+                if (lane == 0 && pw == 0) hbeat(P, 3, ((unsigned long long)(st.k + 1) << 40) | (unsigned long long)recn);
+                if ((int)(recn % NPOLL) != pw || !(R.flags() & REC_FIRST)) continue;
                 const int2 lw = R.lane(lane);
                 const int ne = lw.x >= 0 ? meta_ne((unsigned)lw.y) : 0;
                 if (!__any_sync(0xffffffffu, ne > 0)) continue;
@@ -863,7 +906,7 @@ __device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st
                 for (;;) {                                     // warp-uniform control flow
                     __syncwarp();
                     const long long pmin = __shfl_sync(0xffffffffu, (long long)S.progress[0], 0);
-                    if (lane == 0) { hbeat(P, 6, (unsigned long long)pmin); hbeat(P, 7, it); }
+                    if (lane == 0 && pw == 0) { hbeat(P, 6, (unsigned long long)pmin); hbeat(P, 7, it); }
                     if (pmin >= recn) break;                   // the solver is here: it polls itself
                     if (recn <= pmin + POLL_AHEAD) {           // close enough: values may be there
                         double e = 0.0;
@@ -893,9 +936,10 @@ __device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st
         // ---------------- solver warp (one per CTA)
         const int ncL = (c0 < cu) ? min(cu, c1) - c0 : 0;       // chunks of the L section
         if (lane == 0) trace_mark(P, st.k, 8 + 4 * blockIdx.x + 0);
+        SolveCtx C{S.yring, &S, y, nullptr, P.p, P.mbL, P.sc, ep, pb, mask};
         if (ncL > 0) {
             double dummy = 0.0;
-            solver_section<false, false>(P, S, q0, 0, ncL, rec0, y, nullptr, P.mbL, ep, pb, mask, &dummy);
+            solver_section<false, false>(C, S, q0, 0, ncL, rec0, dummy, P, st.k);
             __syncwarp();
             if (lane == 0 && c1 > cu) {
                 mbar_arrive(S.ldone);                              // y of the L section complete
@@ -905,10 +949,11 @@ __device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st
         if (ncL < nch) {
             long long n = 0;                                        // U records continue the numbering
             for (int t = 0; t < ncL; ++t) n += *(const uint16_t*)(P.stream + (size_t)(c0 + t) * SPCG_CHUNK_BYTES);
-            if (kind == K_PRO)
-                solver_section<true, true>(P, S, q0, ncL, nch, rec0 + n, z, rdot, P.mbU, ep, pb, mask, &rz);
-            else
-                solver_section<true, false>(P, S, q0, ncL, nch, rec0 + n, z, rdot, P.mbU, ep, pb, mask, &rz);
+            C.out = z;
+            C.rdot = rdot;
+            C.mb = P.mbU;
+            if (kind == K_PRO) solver_section<true, true>(C, S, q0, ncL, nch, rec0 + n, rz, P, st.k);
+            else solver_section<true, false>(C, S, q0, ncL, nch, rec0 + n, rz, P, st.k);
         }
         if (lane == 0) trace_mark(P, st.k, 8 + 4 * blockIdx.x + 2);
     }
@@ -1250,7 +1295,7 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         spcg_dev_destroy(d);
         return SPCG_ERR_CUDA;
     }
-    if (getenv("SPCG_TRACE")) {
+    if (getenv("SPCG_HB")) {
         void* hp = nullptr;
         if (cudaHostAlloc(&hp, sizeof(unsigned long long) * 8 * (size_t)lay.parts, cudaHostAllocMapped) == cudaSuccess) {
             memset(hp, 0, sizeof(unsigned long long) * 8 * (size_t)lay.parts);
@@ -1259,6 +1304,8 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
             cudaHostGetDevicePointer(&dp, hp, 0);
             P.hb = (unsigned long long*)dp;
         }
+    }
+    if (getenv("SPCG_TRACE")) {
         void* tp = nullptr;
         if (alloc(d, sizeof(unsigned long long) * (8 + 4 * (size_t)lay.parts + 400), &tp) == SPCG_OK) {
             d->trace = (unsigned long long*)tp;
@@ -1393,4 +1440,18 @@ spcg_status_t spcg_dev_copy(spcg_device_t* d, void* dst, const void* src, size_t
     CK(cudaMemcpyAsync(dst, src, bytes, kind == 1 ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToHost, d->stream));
     CK(cudaStreamSynchronize(d->stream));
     return SPCG_OK;
+}
+
+// debug: slow-path counters (env SPCG_COUNT)
+extern "C" int spcg_dbg_counts(unsigned long long* out) {
+    static unsigned long long* d = nullptr;
+    if (!d) {
+        if (cudaMalloc(&d, 64) != cudaSuccess) return -1;
+        cudaMemset(d, 0, 64);
+        cudaMemcpyToSymbol(g_dbg_counts, &d, sizeof(d));
+        return 0;
+    }
+    cudaMemcpy(out, d, 24, cudaMemcpyDeviceToHost);
+    cudaMemset(d, 0, 64);
+    return 1;
 }

@@ -17,6 +17,12 @@
 #include <algorithm>
 #include <cmath>
 #include <cstring>
+#include <iterator>
+#include <cstdio>
+#include <cstdlib>
+#include <map>
+#include <set>
+#include <string>
 
 #include "internal.h"
 
@@ -191,40 +197,218 @@ static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev,
 }
 
 // ---------------------------------------------------------------- chunked stream
-// Ring-safety of intra-part dependencies for one factor (slot = (row - part_begin) & (ring-1)):
-// entry (i,j) may read j from the shared ring iff no other row of the part that maps to the
-// same slot is written between j's step and i's step (inclusive).
-static void ring_analysis(const Csr& M, bool upper, const std::vector<int32_t>& lev, const std::vector<int64_t>& pb,
-                          int32_t ring, std::vector<int32_t>& part_of, std::vector<int32_t>& step_of,
-                          std::vector<int32_t>& next_writer) {
-    const int64_t n = M.n;
-    const int parts = (int)pb.size() - 1;
-    (void)upper;
-    part_of.assign(n, 0);
+// Partition of the rows over the CTAs (parts) for the chunked executor.
+//
+// Level-balanced affinity partition: wavefront by wavefront (levels of the L
+// solve), every row goes to the part that owns most of its dependencies, but
+// no part takes more than its equal share of that wavefront.  Every wavefront
+// is therefore spread over all CTAs (parallelism), while dependency chains
+// stay inside a CTA where possible (locality: the shared-memory ring instead of
+// a cross-CTA flag).  Rows without dependencies are placed by their position
+// inside the wavefront.  Needs no geometry.
+struct Partition {
+    int parts = 1;
+    std::vector<int32_t> part_of;              // [n]
+    std::vector<int32_t> lidx;                 // [n] index inside the part (ascending rows)
+    std::vector<std::vector<int32_t>> rows;    // per part, ascending
+};
+
+static void partition_level_based(const Factors& F, int P, bool affinity, Partition& out) {
+    const int64_t n = F.L.n;
+    out.parts = P;
+    out.part_of.assign(n, -1);
+    std::vector<int64_t> lp(F.wL + 1, 0);
+    for (int64_t i = 0; i < n; ++i) lp[F.levL[i] + 1]++;
+    for (int64_t l = 0; l < F.wL; ++l) lp[l + 1] += lp[l];
+    std::vector<int32_t> lrows(n);
+    {
+        std::vector<int64_t> nx(lp.begin(), lp.end() - 1);
+        for (int64_t i = 0; i < n; ++i) lrows[nx[F.levL[i]]++] = (int32_t)i;
+    }
+    std::vector<int32_t> load(P, 0), cnt(P, 0), touched;
+    std::vector<int32_t> deferred, target;
+    for (int64_t l = 0; l < F.wL && !affinity; ++l) {   // position-in-wavefront variant
+        // position-in-wavefront: the t-th of m rows (ascending) goes to part floor(t P / m)
+        const int64_t m = lp[l + 1] - lp[l];
+        for (int64_t t = lp[l]; t < lp[l + 1]; ++t) out.part_of[lrows[t]] = (int32_t)(((t - lp[l]) * P) / m);
+    }
+    for (int64_t l = 0; l < F.wL && affinity; ++l) {
+        const int64_t m = lp[l + 1] - lp[l];
+        const int32_t cap = (int32_t)((m + P - 1) / P);
+        std::fill(load.begin(), load.end(), 0);
+        deferred.clear();
+        target.clear();
+        for (int64_t t = lp[l]; t < lp[l + 1]; ++t) {
+            const int32_t i = lrows[t];
+            // part owning most dependencies (ties: the larger dependency row's part)
+            int best = -1, bestc = 0;
+            touched.clear();
+            for (int64_t q = F.L.rp[i]; q < F.L.rp[i + 1]; ++q) {
+                const int pj = out.part_of[F.L.col[q]];
+                if (cnt[pj]++ == 0) touched.push_back(pj);
+                if (cnt[pj] >= bestc) { bestc = cnt[pj]; best = pj; }
+            }
+            for (int pj : touched) cnt[pj] = 0;
+            if (best >= 0 && load[best] < cap) {
+                out.part_of[i] = best;
+                load[best]++;
+            } else {
+                deferred.push_back(i);
+                target.push_back(best >= 0 ? best : (int)(((t - lp[l]) * P) / m));
+            }
+        }
+        // deferred rows: nearest part (by id) with spare capacity
+        std::set<int> open;
+        for (int p = 0; p < P; ++p) if (load[p] < cap) open.insert(p);
+        for (size_t d = 0; d < deferred.size(); ++d) {
+            auto it = open.lower_bound(target[d]);
+            int p;
+            if (it == open.end()) p = *open.rbegin();
+            else if (it == open.begin()) p = *it;
+            else { auto pr = std::prev(it); p = (*it - target[d] <= target[d] - *pr) ? *it : *pr; }
+            out.part_of[deferred[d]] = p;
+            if (++load[p] >= cap) open.erase(p);
+        }
+    }
+    out.rows.assign(P, {});
+    out.lidx.assign(n, 0);
+    for (int64_t i = 0; i < n; ++i) {
+        const int p = out.part_of[i];
+        out.lidx[i] = (int32_t)out.rows[p].size();
+        out.rows[p].push_back((int32_t)i);
+    }
+}
+
+// Contiguous ranges of a row ordering, balanced by per-row work.
+static void partition_contiguous(const Factors& F, int P, const std::vector<int32_t>& ord, Partition& out) {
+    const int64_t n = F.L.n;
+    out.parts = P;
+    out.part_of.assign(n, 0);
+    double tot = 0.0;
+    for (int64_t i = 0; i < n; ++i) tot += 4.0 + (double)(F.L.rp[i + 1] - F.L.rp[i]) + (double)(F.U.rp[i + 1] - F.U.rp[i]);
+    double acc = 0.0;
+    for (int64_t t = 0; t < n; ++t) {
+        const int32_t i = ord[t];
+        const double wi = 4.0 + (double)(F.L.rp[i + 1] - F.L.rp[i]) + (double)(F.U.rp[i + 1] - F.U.rp[i]);
+        out.part_of[i] = std::min(P - 1, (int)((acc + 0.5 * wi) * P / tot));
+        acc += wi;
+    }
+    out.rows.assign(P, {});
+    out.lidx.assign(n, 0);
+    for (int64_t i = 0; i < n; ++i) {
+        const int p = out.part_of[i];
+        out.lidx[i] = (int32_t)out.rows[p].size();
+        out.rows[p].push_back((int32_t)i);
+    }
+}
+
+// Executor model used to pick a partition: every part walks its wavefront groups
+// in order, a slice of <= 32 rows costs t_rec, and a dependency produced by
+// another part is usable H after it was produced.  Returns the modelled time of
+// one forward solve (the backward solve mirrors it).
+static double model_solve_time(const Factors& F, const Partition& PT, double t_rec, double H) {
+    const int64_t n = F.L.n;
+    std::vector<int64_t> lp(F.wL + 1, 0);
+    for (int64_t i = 0; i < n; ++i) lp[F.levL[i] + 1]++;
+    for (int64_t l = 0; l < F.wL; ++l) lp[l + 1] += lp[l];
+    std::vector<int32_t> lrows(n);
+    {
+        std::vector<int64_t> nx(lp.begin(), lp.end() - 1);
+        for (int64_t i = 0; i < n; ++i) lrows[nx[F.levL[i]]++] = (int32_t)i;
+    }
+    std::vector<double> fin(n, 0.0), clock(PT.parts, 0.0), ready(PT.parts, 0.0);
+    std::vector<int32_t> cnt(PT.parts, 0), touched;
+    for (int64_t l = 0; l < F.wL; ++l) {
+        touched.clear();
+        for (int64_t t = lp[l]; t < lp[l + 1]; ++t) {
+            const int32_t i = lrows[t];
+            const int p = PT.part_of[i];
+            if (cnt[p]++ == 0) { touched.push_back(p); ready[p] = clock[p]; }
+            for (int64_t q = F.L.rp[i]; q < F.L.rp[i + 1]; ++q) {
+                const int32_t j = F.L.col[q];
+                if (PT.part_of[j] != p) ready[p] = std::max(ready[p], fin[j] + H);
+            }
+        }
+        for (int p : touched) {
+            clock[p] = ready[p] + t_rec * (double)((cnt[p] + 31) / 32);
+            cnt[p] = 0;
+        }
+        for (int64_t t = lp[l]; t < lp[l + 1]; ++t) fin[lrows[t]] = clock[PT.part_of[lrows[t]]];
+    }
+    return *std::max_element(clock.begin(), clock.end());
+}
+
+// most frequent strictly-lower offset i - j > 1 of L (the grid line length for stencils)
+static int64_t dominant_stride(const Factors& F) {
+    std::map<int64_t, int64_t> h;
+    const int64_t n = F.L.n;
+    const int64_t step = std::max<int64_t>(1, n / 20000);
+    for (int64_t i = 0; i < n; i += step)
+        for (int64_t q = F.L.rp[i]; q < F.L.rp[i + 1]; ++q) {
+            const int64_t d = i - F.L.col[q];
+            if (d > 1) h[d]++;
+        }
+    int64_t best = 0, bc = 0;
+    for (auto& kv : h) if (kv.second > bc) { bc = kv.second; best = kv.first; }
+    return best;
+}
+
+// Inspector: build candidate partitions and keep the one the model says is fastest.
+static void partition_rows(const Factors& F, int P, Partition& out, std::string* chosen) {
+    const int64_t n = F.L.n;
+    const double T_REC = 0.45, H = 1.0;          // microseconds, measured on B200
+    std::vector<std::pair<std::string, Partition>> cand;
+    std::vector<int32_t> ord(n);
+    for (int64_t i = 0; i < n; ++i) ord[i] = (int32_t)i;
+    { Partition p; partition_contiguous(F, P, ord, p); cand.push_back({"contiguous", std::move(p)}); }
+    const int64_t s = dominant_stride(F);
+    if (s > 1 && s < n) {
+        // rows ordered by (i mod s, i / s): contiguous ranges become strips across the stride
+        std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return a % s < b % s; });
+        Partition p;
+        partition_contiguous(F, P, ord, p);
+        cand.push_back({"strided", std::move(p)});
+    }
+    { Partition p; partition_level_based(F, P, true, p); cand.push_back({"affinity", std::move(p)}); }
+    const char* force = getenv("SPCG_PART");
+    double best = 1e300;
+    size_t bi = 0;
+    for (size_t c = 0; c < cand.size(); ++c) {
+        const double t = model_solve_time(F, cand[c].second, T_REC, H);
+        if (getenv("SPCG_PART_VERBOSE")) fprintf(stderr, "[spcg] partition %s: modelled forward solve %.1f us\n", cand[c].first.c_str(), t);
+        if (force ? cand[c].first == force : t < best) { best = force ? 0.0 : t; bi = c; }
+    }
+    out = std::move(cand[bi].second);
+    if (chosen) *chosen = cand[bi].first;
+}
+
+// Ring-safety of intra-part dependencies for one factor (slot = lidx & (ring-1)):
+// entry (i,j) may read j from the shared ring iff no other row of the part that
+// maps to the same slot is written between j's step and i's step (inclusive).
+static void ring_analysis(const Partition& PT, const std::vector<int32_t>& lev, int32_t ring,
+                          std::vector<int32_t>& step_of, std::vector<int32_t>& next_writer) {
+    const int64_t n = (int64_t)PT.part_of.size();
     step_of.assign(n, 0);
     next_writer.assign(n, INT32_MAX);
-    for (int c = 0; c < parts; ++c) {
-        int32_t lmin = INT32_MAX;
-        for (int64_t i = pb[c]; i < pb[c + 1]; ++i) { part_of[i] = c; lmin = std::min(lmin, lev[i]); }
-        // steps = dense rank of the levels present in the part
-        std::vector<int32_t> lv;
-        for (int64_t i = pb[c]; i < pb[c + 1]; ++i) lv.push_back(lev[i]);
+    std::vector<int32_t> lv;
+    std::vector<std::pair<int32_t, int32_t>> mem;
+    for (int c = 0; c < PT.parts; ++c) {
+        const std::vector<int32_t>& R = PT.rows[c];
+        lv.clear();
+        for (int32_t i : R) lv.push_back(lev[i]);
         std::sort(lv.begin(), lv.end());
         lv.erase(std::unique(lv.begin(), lv.end()), lv.end());
-        for (int64_t i = pb[c]; i < pb[c + 1]; ++i)
-            step_of[i] = (int32_t)(std::lower_bound(lv.begin(), lv.end(), lev[i]) - lv.begin());
-        const int64_t sz = pb[c + 1] - pb[c];
-        if (sz <= ring) continue;
-        std::vector<std::pair<int32_t, int32_t>> mem;
+        for (int32_t i : R) step_of[i] = (int32_t)(std::lower_bound(lv.begin(), lv.end(), lev[i]) - lv.begin());
+        if ((int64_t)R.size() <= ring) continue;
         for (int64_t cls = 0; cls < ring; ++cls) {
             mem.clear();
-            for (int64_t j = pb[c] + cls; j < pb[c + 1]; j += ring) mem.push_back({step_of[j], (int32_t)j});
+            for (int64_t t = cls; t < (int64_t)R.size(); t += ring) mem.push_back({step_of[R[t]], R[t]});
             if (mem.size() < 2) continue;
             std::sort(mem.begin(), mem.end());
             for (size_t a = 0; a < mem.size();) {
                 size_t b = a;
                 while (b < mem.size() && mem[b].first == mem[a].first) ++b;
-                int32_t nxt = (b - a > 1) ? mem[a].first : (b < mem.size() ? mem[b].first : INT32_MAX);
+                const int32_t nxt = (b - a > 1) ? mem[a].first : (b < mem.size() ? mem[b].first : INT32_MAX);
                 for (size_t t = a; t < b; ++t) next_writer[mem[t].second] = nxt;
                 a = b;
             }
@@ -242,7 +426,7 @@ struct StreamWriter {
         if (cur >= 0) finish();
         cur = (int64_t)(S.bytes.size() / SPCG_CHUNK_BYTES);
         S.bytes.resize(S.bytes.size() + SPCG_CHUNK_BYTES, 0);
-        used = 16;
+        used = SPCG_CHUNK_HDR;
         nrec = 0;
     }
     void finish() {
@@ -258,6 +442,8 @@ struct StreamWriter {
     uint8_t* alloc(int32_t bytes, uint8_t& side) {
         if (cur < 0 || used + bytes > SPCG_CHUNK_BYTES || nrec == SPCG_MAXREC) new_chunk();
         uint8_t* p = &S.bytes[cur * SPCG_CHUNK_BYTES + used];
+        uint16_t off = (uint16_t)used;
+        std::memcpy(&S.bytes[cur * SPCG_CHUNK_BYTES + 8 + 2 * nrec], &off, 2);   // record offset table
         used += bytes;
         side = (uint8_t)nrec++;
         S.records++;
@@ -270,15 +456,14 @@ void put(uint8_t* base, size_t off, T v) { std::memcpy(base + off, &v, sizeof(T)
 }  // namespace
 
 // one phase (L or U) of one part into the stream
-static void emit_section(StreamWriter& W, const Csr& M, bool upper, const std::vector<int32_t>& lev, int64_t lo,
-                         int64_t hi, const std::vector<int32_t>& part_of, const std::vector<int32_t>& step_of,
-                         const std::vector<int32_t>& next_writer, const std::vector<uint8_t>& publish, int64_t pbc,
-                         int32_t ring, bool sync_first) {
-    if (hi <= lo) return;
+static void emit_section(StreamWriter& W, const Csr& M, bool upper, const std::vector<int32_t>& lev,
+                         const std::vector<int32_t>& prow, const Partition& PT, const std::vector<int32_t>& step_of,
+                         const std::vector<int32_t>& next_writer, const std::vector<uint8_t>& publish, int32_t ring,
+                         bool sync_first) {
+    if (prow.empty()) return;
     auto dep_begin = [&](int64_t i) { return upper ? M.rp[i] + 1 : M.rp[i]; };
     // rows of the part grouped by level (ascending), rows ascending inside a level
-    std::vector<int32_t> order;
-    for (int64_t i = lo; i < hi; ++i) order.push_back((int32_t)i);
+    std::vector<int32_t> order(prow.begin(), prow.end());
     std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return lev[a] < lev[b]; });
     int prev_ns = -1;
     bool first_record = true;
@@ -303,9 +488,9 @@ static void emit_section(StreamWriter& W, const Csr& M, bool upper, const std::v
                 for (int pass = 0; pass < 2; ++pass)
                     for (int64_t q = dep_begin(r); q < M.rp[r + 1]; ++q) {
                         const int32_t j = M.col[q];
-                        const bool safe = part_of[j] == part_of[r] && next_writer[j] > step_of[r];
+                        const bool safe = PT.part_of[j] == PT.part_of[r] && next_writer[j] > step_of[r];
                         if ((pass == 0) == safe) continue;
-                        esrc[l].push_back(safe ? (int32_t)((j - pbc) & (ring - 1)) : -j - 1);
+                        esrc[l].push_back(safe ? (int32_t)(PT.lidx[j] & (ring - 1)) : -j - 1);
                         evalv[l].push_back(M.val[q]);
                     }
                 ne_tot[l] = 0;
@@ -342,12 +527,14 @@ static void emit_section(StreamWriter& W, const Csr& M, bool upper, const std::v
                 for (int l = 0; l < 32; ++l) {
                     const int32_t r = l < m ? order[s0 + l] : -1;
                     int len = 0, ne = 0;
+                    uint32_t dst = 0;
                     if (l < m) {
                         len = std::max(0, std::min<int>(wp, (int)esrc[l].size() - k0));
                         ne = std::max(0, std::min<int>(len, ne_tot[l] - k0));
+                        dst = (uint32_t)(PT.lidx[r] & (ring - 1));
                     }
-                    // lane word: {row, meta = len | ne << 8 | publish << 16}
-                    const uint32_t meta = (uint32_t)len | ((uint32_t)ne << 8) | (((pub >> l) & 1u) << 16);
+                    // lane word: {row, meta = len | ne << 8 | publish << 16 | ring slot << 17}
+                    const uint32_t meta = (uint32_t)len | ((uint32_t)ne << 8) | (((pub >> l) & 1u) << 16) | (dst << 17);
                     put<int32_t>(rec, 16 + 8 * l, r);
                     put<uint32_t>(rec, 20 + 8 * l, meta);
                     for (int k = 0; k < len; ++k) {
@@ -365,21 +552,21 @@ static void emit_section(StreamWriter& W, const Csr& M, bool upper, const std::v
     }
 }
 
-static void build_chunk_stream(const Factors& F, const std::vector<int64_t>& pb, int32_t ring, ChunkStream& S) {
+static void build_chunk_stream(const Factors& F, const Partition& PT, int32_t ring, ChunkStream& S) {
     const int64_t n = F.L.n;
-    const int parts = (int)pb.size() - 1;
-    std::vector<int32_t> partL, stepL, nwL, partU, stepU, nwU;
-    ring_analysis(F.L, false, F.levL, pb, ring, partL, stepL, nwL);
-    ring_analysis(F.U, true, F.levU, pb, ring, partU, stepU, nwU);
+    const int parts = PT.parts;
+    std::vector<int32_t> stepL, nwL, stepU, nwU;
+    ring_analysis(PT, F.levL, ring, stepL, nwL);
+    ring_analysis(PT, F.levU, ring, stepU, nwU);
     std::vector<uint8_t> pubL(n, 0), pubU(n, 0);
     for (int64_t i = 0; i < n; ++i) {
         for (int64_t q = F.L.rp[i]; q < F.L.rp[i + 1]; ++q) {
             const int32_t j = F.L.col[q];
-            if (!(partL[j] == partL[i] && nwL[j] > stepL[i])) pubL[j] = 1;
+            if (!(PT.part_of[j] == PT.part_of[i] && nwL[j] > stepL[i])) pubL[j] = 1;
         }
         for (int64_t q = F.U.rp[i] + 1; q < F.U.rp[i + 1]; ++q) {
             const int32_t j = F.U.col[q];
-            if (!(partU[j] == partU[i] && nwU[j] > stepU[i])) pubU[j] = 1;
+            if (!(PT.part_of[j] == PT.part_of[i] && nwU[j] > stepU[i])) pubU[j] = 1;
         }
     }
     S = ChunkStream();
@@ -389,10 +576,10 @@ static void build_chunk_stream(const Factors& F, const std::vector<int64_t>& pb,
     for (int c = 0; c < parts; ++c) {
         W.new_chunk();
         S.part_chunk[c] = (int32_t)W.cur;
-        emit_section(W, F.L, false, F.levL, pb[c], pb[c + 1], partL, stepL, nwL, pubL, pb[c], ring, false);
+        emit_section(W, F.L, false, F.levL, PT.rows[c], PT, stepL, nwL, pubL, ring, false);
         W.new_chunk();                     // U section starts on a chunk boundary
         S.part_uchunk[c] = (int32_t)W.cur;
-        emit_section(W, F.U, true, F.levU, pb[c], pb[c + 1], partU, stepU, nwU, pubU, pb[c], ring, true);
+        emit_section(W, F.U, true, F.levU, PT.rows[c], PT, stepU, nwU, pubU, ring, true);
     }
     W.finish();
     S.part_chunk[parts] = (int32_t)(S.bytes.size() / SPCG_CHUNK_BYTES);
@@ -405,33 +592,22 @@ void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, 
     out.parts = parts;
     out.part_begin.assign(parts + 1, 0);
     if (strategy == SPCG_SPTRSV_CHUNKED) {
-        // contiguous row ranges balanced by per-row work (rows + factor entries)
-        std::vector<double> pre(n + 1, 0.0);
-        for (int64_t i = 0; i < n; ++i)
-            pre[i + 1] = pre[i] + 4.0 + (double)(F.L.rp[i + 1] - F.L.rp[i]) + (double)(F.U.rp[i + 1] - F.U.rp[i]);
-        int64_t r = 0;
-        for (int c = 1; c < parts; ++c) {
-            double target = pre[n] * c / parts;
-            while (r < n && pre[r] < target) ++r;
-            out.part_begin[c] = r;
-        }
-        out.part_begin[parts] = n;
-        int64_t maxsz = 0;
-        for (int c = 0; c < parts; ++c) maxsz = std::max(maxsz, out.part_begin[c + 1] - out.part_begin[c]);
+        Partition PT;
+        partition_rows(F, parts, PT, &out.partition);
+        size_t maxsz = 1;
+        for (int c = 0; c < parts; ++c) maxsz = std::max(maxsz, PT.rows[c].size());
         int32_t ring = 1;
-        while (ring < maxsz && ring < ring_max) ring <<= 1;
+        while ((size_t)ring < maxsz && ring < ring_max) ring <<= 1;
         out.ring = ring;
-    } else {
-        out.part_begin[parts] = n;
-        out.ring = 0;
+        for (int c = 0; c < parts; ++c) out.part_begin[c + 1] = out.part_begin[c] + (int64_t)PT.rows[c].size();
+        build_chunk_stream(F, PT, ring, out.S);
+        return;
     }
-    std::vector<int64_t> pb = strategy == SPCG_SPTRSV_CHUNKED ? out.part_begin : std::vector<int64_t>{0, n};
-    if (strategy == SPCG_SPTRSV_CHUNKED) {
-        build_chunk_stream(F, pb, out.ring, out.S);
-    } else {
-        build_tri(F.L, false, F.levL, F.wL, strategy, pb, out.ring, out.L);
-        build_tri(F.U, true, F.levU, F.wU, strategy, pb, out.ring, out.U);
-    }
+    out.part_begin[parts] = n;
+    out.ring = 0;
+    const std::vector<int64_t> pb{0, n};
+    build_tri(F.L, false, F.levL, F.wL, strategy, pb, out.ring, out.L);
+    build_tri(F.U, true, F.levU, F.wU, strategy, pb, out.ring, out.U);
 }
 
 }  // namespace spcg
