@@ -274,22 +274,59 @@ __device__ void global_sums(const double* partials, int slot_a, int slot_b, doub
 }
 
 // ------------------------------------------------------------------ phases
-// w = A p (SELL-32, thread per row) and the partial (p, w)
+// w = A p (SELL-32, thread per row) and the partial (p, w).  A warp takes SU
+// consecutive slices per step and issues all their index/value loads, then all
+// gathers of p, then the FMA chains (k ascending per row, as the definition):
+// SU x SK independent loads in flight instead of one dependent chain.
+constexpr int SU = 4, SK = 4;
 __device__ void phase_spmv(const Params& P, const double* pin, double* wout, double& pw) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int64_t W = (int64_t)gridDim.x * NWARP;
-    for (int64_t s = (int64_t)blockIdx.x * NWARP + warp; s < P.A.nslices; s += W) {
-        const int64_t e0 = P.A.eoff[s];
-        const int wd = (int)(P.A.eoff[s + 1] - e0);
-        const int32_t* cp = P.A.col + e0 * 32 + lane;
-        const double* vp = P.A.val + e0 * 32 + lane;
-        double acc = 0.0;
-#pragma unroll 4
-        for (int k = 0; k < wd; ++k) acc = fma(__ldg(vp + 32 * k), pin[__ldg(cp + 32 * k)], acc);
-        const int64_t row = s * 32 + lane;
-        if (row < P.n) {
-            wout[row] = acc;
-            pw = fma(pin[row], acc, pw);
+    const int64_t ns = P.A.nslices;
+    const int64_t stride = (int64_t)gridDim.x * NWARP * SU;
+    for (int64_t s0 = ((int64_t)blockIdx.x * NWARP + warp) * SU; s0 < ns; s0 += stride) {
+        const int64_t eo = (lane <= SU && s0 + lane <= ns) ? __ldg(P.A.eoff + s0 + lane) : 0;
+        int64_t e[SU];
+        int wd[SU];
+        int wmax = 0;
+#pragma unroll
+        for (int u = 0; u < SU; ++u) {
+            e[u] = __shfl_sync(0xffffffffu, eo, u);
+            const int64_t e1 = __shfl_sync(0xffffffffu, eo, u + 1);
+            wd[u] = (s0 + u < ns) ? (int)(e1 - e[u]) : 0;
+            wmax = max(wmax, wd[u]);
+        }
+        double acc[SU];
+#pragma unroll
+        for (int u = 0; u < SU; ++u) acc[u] = 0.0;
+        for (int kb = 0; kb < wmax; kb += SK) {
+            int c[SU][SK];
+            double v[SU][SK], g[SU][SK];
+#pragma unroll
+            for (int u = 0; u < SU; ++u)
+#pragma unroll
+                for (int k = 0; k < SK; ++k) {
+                    const bool on = kb + k < wd[u];
+                    const int64_t idx = (e[u] + kb + k) * 32 + lane;
+                    c[u][k] = on ? __ldg(P.A.col + idx) : 0;
+                    v[u][k] = on ? __ldg(P.A.val + idx) : 0.0;
+                }
+#pragma unroll
+            for (int u = 0; u < SU; ++u)
+#pragma unroll
+                for (int k = 0; k < SK; ++k) g[u][k] = pin[c[u][k]];
+#pragma unroll
+            for (int u = 0; u < SU; ++u)
+#pragma unroll
+                for (int k = 0; k < SK; ++k)
+                    if (kb + k < wd[u]) acc[u] = fma(v[u][k], g[u][k], acc[u]);
+        }
+#pragma unroll
+        for (int u = 0; u < SU; ++u) {
+            const int64_t row = (s0 + u) * 32 + lane;
+            if (s0 + u < ns && row < P.n) {
+                wout[row] = acc[u];
+                pw = fma(pin[row], acc[u], pw);
+            }
         }
     }
 }
