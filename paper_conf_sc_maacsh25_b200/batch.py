@@ -1,0 +1,120 @@
+"""Multi-GPU batch of independent systems.
+
+A single system does not shard (the triangular-solve chain is serial across
+wavefronts), so multi-GPU use is data-parallel over *independent systems*: the
+batch is split across ranks by LPT (longest processing time first) on a cost
+estimate, every rank sets up and solves its own systems on its own GPU, and the
+only communication is a host-side gather of the per-system results (no
+collective on the solve path).  Launch one process per GPU (torchrun); ranks use
+``torch.distributed`` only for the final gather and the timing barrier.
+"""
+from __future__ import annotations
+
+import math
+import time
+from dataclasses import dataclass, field
+
+import numpy as np
+
+import gen
+
+from . import SPCG
+
+
+@dataclass
+class System:
+    index: int
+    family: str
+    params: tuple
+    K: int
+    cost: float = 0.0
+
+
+def batch_systems(count: int = 64):
+    """C5: system i of the seeded mixed batch."""
+    out = []
+    for i in range(count):
+        s = gen.batch_spec(i)
+        out.append(System(i, s["family"], tuple(s["params"]), s["K"]))
+    return out
+
+
+def estimate_cost(s: System) -> float:
+    """Relative solve cost ~ bytes per iteration x expected iterations.
+
+    Rows from the grid sides; stored entries per row by stencil (x ~2.5 for
+    ILU(2) fill); iterations ~ grid side (CG on Laplacian-like systems)."""
+    dims = [p for p in s.params if isinstance(p, (int, np.integer))][: 3 if s.family in ("poisson3d", "fem_q1") else 2]
+    n = float(np.prod(dims))
+    per_row = {"poisson2d": 5, "aniso_layered": 5, "poisson3d": 7, "fem_q1": 27}[s.family]
+    fill = 2.5 if s.K >= 2 else 1.0
+    side = max(dims)
+    return n * (12.0 * per_row * (1.0 + fill) + 120.0) * side
+
+
+def lpt_assign(systems, world: int):
+    """Longest-processing-time-first: each system (largest cost first) goes to the
+    currently least-loaded rank.  Deterministic (ties: lowest rank, then index)."""
+    for s in systems:
+        if s.cost == 0.0:
+            s.cost = estimate_cost(s)
+    order = sorted(systems, key=lambda s: (-s.cost, s.index))
+    load = [0.0] * world
+    plan = [[] for _ in range(world)]
+    for s in order:
+        r = min(range(world), key=lambda k: (load[k], k))
+        plan[r].append(s)
+        load[r] += s.cost
+    for p in plan:
+        p.sort(key=lambda s: s.index)
+    return plan, load
+
+
+@dataclass
+class Result:
+    index: int
+    family: str
+    n: int
+    iterations: int = 0
+    iter_phase_ms: float = 0.0
+    rnorm: float = 0.0
+    status: int = 0
+    chosen_pct: float = 0.0
+    levels_L: int = 0
+    x_checksum: float = 0.0
+    setup_s: float = 0.0
+
+
+def setup_rank(systems, device: int, mode: str = "alg2", **kw):
+    """Host setup (+ upload when device >= 0) of this rank's systems."""
+    handles = []
+    for s in systems:
+        A = gen.make(s.family, *s.params)
+        b, _ = gen.rhs(A)
+        t0 = time.perf_counter()
+        h = SPCG(A, mode=mode, K=s.K, device=device, **kw)
+        handles.append((s, A, b, h, time.perf_counter() - t0))
+    return handles
+
+
+def solve_rank(handles, eps: float = 1e-8, kmax: int = 20000):
+    """Solve this rank's systems on its GPU; returns per-system results."""
+    import torch
+    out = []
+    for s, A, b, h, st in handles:
+        bd = torch.from_numpy(b).to(f"cuda:{h.device}")
+        x, info = h.solve(bd, eps=eps, kmax=kmax)
+        out.append(Result(s.index, s.family, A.n, info["iterations"], info["iter_phase_ms"], info["rnorm"],
+                          info["status"], h.info["chosen_pct"], h.info["levels_L"],
+                          float(x.double().sum().item()), st))
+    return out
+
+
+def gather(results, world: int):
+    """Host-side gather of every rank's results onto all ranks (gloo or nccl)."""
+    if world == 1:
+        return sorted(results, key=lambda r: r.index)
+    import torch.distributed as dist
+    allr = [None] * world
+    dist.all_gather_object(allr, results)
+    return sorted([r for part in allr for r in part], key=lambda r: r.index)
