@@ -197,6 +197,26 @@ spcg_status_t spcg_export(spcg_handle_t h, int32_t what, void* buf, size_t* byte
 
 void spcg_destroy(spcg_handle_t h);
 
+/* Chain-floor calibration: the cost of each handoff a
+ * wavefront executor can put on its critical path — P:L258-261 (Fig. 1 caption:
+ * wavefront barriers "under-utilize GPU resources") — measured on `device`
+ * with %globaltimer.  chain_floor = (levels_L + levels_U) x the handoff the
+ * executor actually uses.  Times in ns; no handle needed; ~0.1 s of GPU time.
+ * Errors: SPCG_ERR_INVALID_ARG (out == NULL), SPCG_ERR_CUDA (detail in
+ * spcg_last_error()). */
+typedef struct {
+    double grid_sync_ns;        /* grid-wide barrier, one 256-thread CTA per SM (LEVEL, per wavefront) */
+    double graph_kernel_ns;     /* kernel-to-kernel latency inside a CUDA graph (a launch per wavefront) */
+    double flag_same_die_ns;    /* one-way release-store -> acquire-spin handoff, CTA pair on one die */
+    double flag_cross_die_ns;   /* the same across the two dies */
+    double syncthreads_ns;      /* __syncthreads, 256 threads */
+    double cluster_sync_ns;     /* barrier.cluster arrive.release + wait.acquire, cluster of 2 */
+    double sm_clock_mhz;        /* cudaDevAttrClockRate */
+    int32_t sms;
+    int32_t flag_pairs_near;    /* CTA pairs classified as same-die (of sms - 1) */
+} spcg_calib_t;
+spcg_status_t spcg_calibrate(int32_t device, spcg_calib_t* out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -19,7 +19,7 @@ import numpy as np
 
 from . import _build
 
-_LIB_PATH = _build.LIB
+_LIB_PATH = os.environ.get("SPCG_LIB", _build.LIB)   # SPCG_LIB: an experiment variant of the same library
 _lib = None
 
 OK, NOT_CONVERGED = 0, 1
@@ -85,7 +85,8 @@ class SolveInfo(ctypes.Structure):
 
 EXPORTED = ["spcg_abi_version", "spcg_status_string", "spcg_last_error", "spcg_drop_params_default",
             "spcg_options_default", "spcg_setup", "spcg_get_setup_info", "spcg_solve", "spcg_apply_spmv",
-            "spcg_apply_lower", "spcg_apply_upper", "spcg_apply_precond", "spcg_export", "spcg_destroy"]
+            "spcg_apply_lower", "spcg_apply_upper", "spcg_apply_precond", "spcg_export", "spcg_destroy",
+            "spcg_calibrate"]
 
 
 def load(path: str | None = None):
@@ -123,10 +124,26 @@ def load(path: str | None = None):
     lib.spcg_export.restype = I32
     lib.spcg_destroy.argtypes = [V]
     lib.spcg_destroy.restype = None
+    lib.spcg_calibrate.argtypes = [I32, ctypes.POINTER(Calib)]
+    lib.spcg_calibrate.restype = I32
     if lib.spcg_abi_version() != 1:
         raise ImportError("libspcg ABI version mismatch")
     _lib = lib
     return lib
+
+
+class Calib(ctypes.Structure):
+    _fields_ = [("grid_sync_ns", ctypes.c_double), ("graph_kernel_ns", ctypes.c_double),
+                ("flag_same_die_ns", ctypes.c_double), ("flag_cross_die_ns", ctypes.c_double),
+                ("syncthreads_ns", ctypes.c_double), ("cluster_sync_ns", ctypes.c_double),
+                ("sm_clock_mhz", ctypes.c_double), ("sms", ctypes.c_int32), ("flag_pairs_near", ctypes.c_int32)]
+
+
+def calibrate(device: int = 0) -> dict:
+    """spcg_calibrate: handoff costs for the chain floor."""
+    c = Calib()
+    _check(load().spcg_calibrate(device, ctypes.byref(c)), "spcg_calibrate")
+    return {f: getattr(c, f) for f, _ in Calib._fields_}
 
 
 def _check(st, what=""):

@@ -28,16 +28,19 @@ def stale() -> bool:
     return any(os.path.getmtime(s) > t for s in _sources())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not stale():
+def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
+    """defines/out: experiment variants (e.g. -DSPCG_VGROUP=1 -> libspcg_v1.so, loaded
+    with SPCG_LIB=...); the default build is libspcg.so."""
+    lib = out or LIB
+    if not force and not defines and out is None and not stale():
         return LIB
-    bdir = os.path.join(HERE, "build")
+    bdir = os.path.join(HERE, "build" if not defines else "build_" + "_".join(d.strip("-D").replace("=", "") for d in defines))
     os.makedirs(bdir, exist_ok=True)
     objs = []
     for cu in sorted(glob.glob(os.path.join(CSRC, "*.cu"))):
         o = os.path.join(bdir, os.path.basename(cu) + ".o")
         cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
-               "-I", os.path.join(ROOT, "include"), "-c", cu, "-o", o]
+               "-I", os.path.join(ROOT, "include"), *defines, "-c", cu, "-o", o]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"nvcc failed:\n{r.stderr}")
@@ -52,11 +55,11 @@ def build(force: bool = False, verbose: bool = False) -> str:
                "-I", os.path.join(ROOT, "include"), "-I", "/usr/local/cuda/include", "-c", cpp, "-o", o]
         subprocess.check_call(cmd)
         objs.append(o)
-    tmp = LIB + ".tmp"
+    tmp = lib + ".tmp"
     cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-Xcompiler", "-fopenmp", "-lgomp"]
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":

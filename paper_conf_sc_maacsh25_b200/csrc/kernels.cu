@@ -430,10 +430,19 @@ constexpr int NVEC = 4;
 constexpr int SOLVER_WARP0 = VEC_WARP0 + NVEC;
 static_assert(SOLVER_WARP0 + SPCG_NSOLVER == NWARP, "warp roles must fill the CTA");
 constexpr int POLL_AHEAD = 8;                     // records
+#ifndef SPCG_VGROUP
+#define SPCG_VGROUP 4
+#endif
+constexpr int VGROUP = SPCG_VGROUP;               // chunks a vector warp serves per round
+constexpr int VBATCH = 4;                         // records whose loads are in flight together
+constexpr int VLIST = (VGROUP * SPCG_MAXREC + NVEC - 1) / NVEC;
+static_assert(VGROUP >= 1 && VGROUP <= SPCG_NCHUNK, "vector group must fit the ring");
 constexpr int SIDE_BYTES = 3 * 256 + 16;          // vec[32], aux[32], ext[32], ext mask
 constexpr size_t CH_RING_BYTES = (size_t)SPCG_NCHUNK * SPCG_CHUNK_BYTES;
 constexpr size_t CH_SIDE_BYTES = (size_t)SPCG_NCHUNK * SPCG_MAXREC * SIDE_BYTES;
 constexpr size_t CH_BAR_BYTES = 512;
+static_assert((3 * SPCG_NCHUNK + 1 + SPCG_NSOLVER + 1) <= 32 && 256 + 2 * NVEC * VLIST <= CH_BAR_BYTES,
+              "barrier block layout");
 
 __host__ __device__ constexpr size_t chunked_smem_bytes(int ring) {
     return (size_t)ring * 8 + CH_RING_BYTES + CH_SIDE_BYTES + CH_BAR_BYTES;
@@ -448,6 +457,7 @@ struct ChunkSmem {
     uint64_t* empty;       // [NCHUNK] solvers + poller done
     uint64_t* ldone;       // solvers finished the L section
     volatile long long* progress;   // [NSOLVER] record index each solver warp is at
+    uint16_t* vlist;       // [NVEC][VLIST] per vector warp: (slot, record) of its records in a group
 };
 
 struct PipeState {         // identical sequence in every role
@@ -520,6 +530,7 @@ __device__ ChunkSmem chunk_smem(double* dyn, int ring) {
     S.empty = bars + 2 * SPCG_NCHUNK;
     S.ldone = bars + 3 * SPCG_NCHUNK;
     S.progress = (volatile long long*)(bars + 3 * SPCG_NCHUNK + 1);
+    S.vlist = (uint16_t*)(bars + 32);
     return S;
 }
 
@@ -791,6 +802,7 @@ __device__ __forceinline__ void solve_record(const SolveCtx& C, const Prep& X, i
             rz = o.y;
         }
     } else {
+        if (g_dbg_counts && lane == 0) atomicAdd(g_dbg_counts + 6, 1ull);
         const double2 o = slow_record<UPPER, PRO>(X.p, X.fl, X.wd, X.row, X.meta, X.r, X.vec, X.aux, acc_carry, rz,
                                                   side_vec(*C.S, slot, X.r), C.yring, C.out, C.rdot, C.pvec, C.mb,
                                                   C.sc, C.ep, C.pb, C.mask);
@@ -809,10 +821,15 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
                                                long long recn, double& rz, const Params& P, long long kk) {
     const int lane = threadIdx.x & 31;
     double acc_carry = 0.0;
+    unsigned long long* dbg = g_dbg_counts;     // debug (SPCG_COUNT): solver wait / busy cycles
+    long long t_wait = 0, t_sec = dbg ? clock64() : 0;
+    const long long recn0 = recn;
     for (int i = ib; i < ie; ++i) {
         const unsigned q = q0 + i;
         const int slot = q % SPCG_NCHUNK;
+        const long long tw = dbg ? clock64() : 0;
         if (!warp_ok(mbar_wait(&S.vfull[slot], (q / SPCG_NCHUNK) & 1, C.sc))) return;
+        if (dbg) t_wait += clock64() - tw;
         const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
         const int nrec = *(const uint16_t*)ch;
         Prep A, B;
@@ -833,6 +850,11 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
         recn += nrec;
         __syncwarp();
         if (lane == 0) mbar_arrive(&S.empty[slot]);
+    }
+    if (dbg && lane == 0) {
+        atomicAdd(dbg + 3, (unsigned long long)t_wait);
+        atomicAdd(dbg + 4, (unsigned long long)(clock64() - t_sec));
+        atomicAdd(dbg + 5, (unsigned long long)(recn - recn0));
     }
 }
 
@@ -871,54 +893,109 @@ __device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st
             if (!ok) break;
         }
     } else if (warp >= VEC_WARP0 && warp < SOLVER_WARP0) {
+        // Chunks are taken in groups of up to VGROUP (never straddling the L/U
+        // boundary); this warp's records of the whole group are listed first and
+        // then served VBATCH at a time with every global load of the batch issued
+        // before the first use, so a group costs ~one memory latency instead of
+        // one per chunk.  VGROUP <= SPCG_NCHUNK: the producer can fill the whole
+        // group without any slot being released, so the wait cannot deadlock.
         const int v = warp - VEC_WARP0;
         bool waited_ldone = false;
         long long recn = rec0;
-        for (int i = 0; i < nch; ++i) {
-            const unsigned q = q0 + i, slot = q % SPCG_NCHUNK, use = q / SPCG_NCHUNK;
-            if (c0 + i >= cu && !waited_ldone && cu > c0) {   // y of the L section must be complete
+        uint16_t* mine = S.vlist + v * VLIST;
+        for (int i0 = 0; i0 < nch;) {
+            int i1 = min(nch, i0 + VGROUP);
+            if (c0 + i0 < cu && c0 + i1 > cu) i1 = cu - c0;
+            if (c0 + i0 >= cu && !waited_ldone && cu > c0) {   // y of the L section must be complete
                 if (!warp_ok(mbar_wait(S.ldone, st.ldone_uses & 1, P.sc))) break;
                 waited_ldone = true;
             }
-            if (v == 0 && lane == 0) hbeat(P, 1, ((unsigned long long)(st.k + 1) << 40) | q);
-            if (!warp_ok(mbar_wait(&S.full[slot], use & 1, P.sc))) break;
-            const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
-            const int nrec = *(const uint16_t*)ch;
-            // records are dealt to the vector warps by their global index (<= 1 per warp per chunk)
-            for (int r = 0; r < nrec; ++r, ++recn) {
-                if ((int)(recn % NVEC) != v) continue;
-                const Rec R(ch + *(const uint16_t*)(ch + 8 + 2 * r));
-                if (!(R.flags() & REC_FIRST)) continue;
-                const int row = R.row(lane);
-                double* vec = side_vec(S, slot, r);
-                if (row >= 0) {
-                    if (!(R.flags() & REC_UPPER)) {
-                        double ri;
-                        if (kind == K_ITER) {                  // all four loads before any store
-                            const double r0 = P.r[row], w0 = P.w[row], x0 = P.x[row], p0 = P.p[row];
-                            ri = r0 - alpha * w0;
-                            P.r[row] = ri;
-                            P.x[row] = x0 + alpha * p0;
-                        } else {
-                            ri = rin[row];
-                            if (kind == K_PRO) {
-                                if (rin != P.r) P.r[row] = ri;
-                                if (!P.use_x0) P.x[row] = 0.0;
-                            }
-                        }
-                        rr = fma(ri, ri, rr);
-                        vec[lane] = ri;
-                    } else {
-                        const double y0 = __ldcg(yin + row);
-                        const double a0 = rdot ? __ldcg(rdot + row) : 0.0;
-                        vec[lane] = y0;
-                        side_aux(S, slot, r)[lane] = a0;
-                    }
+            if (v == 0 && lane == 0) hbeat(P, 1, ((unsigned long long)(st.k + 1) << 40) | (q0 + i0));
+            bool ok = true;
+            for (int i = i0; i < i1 && ok; ++i) {
+                const unsigned q = q0 + i;
+                ok = mbar_wait(&S.full[q % SPCG_NCHUNK], (q / SPCG_NCHUNK) & 1, P.sc);
+            }
+            if (!warp_ok(ok)) break;
+            // list: records are dealt to the vector warps by their global index
+            int cnt = 0;
+            for (int i = i0; i < i1; ++i) {
+                const unsigned slot = (q0 + i) % SPCG_NCHUNK;
+                const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
+                const int nrec = *(const uint16_t*)ch;
+                for (int r = 0; r < nrec; ++r, ++recn) {
+                    if ((int)(recn % NVEC) != v) continue;
+                    if (!(*(const uint16_t*)(ch + *(const uint16_t*)(ch + 8 + 2 * r) + 2) & REC_FIRST)) continue;
+                    if (lane == 0) mine[cnt] = (uint16_t)(slot * SPCG_MAXREC + r);
+                    ++cnt;
                 }
-                if (lane == 0) *side_mask(S, slot, r) = 0u;
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&S.vfull[slot]);
+            for (int b0 = 0; b0 < cnt; b0 += VBATCH) {
+                int row[VBATCH], e[VBATCH], fl[VBATCH];
+                double l0[VBATCH], l1[VBATCH], l2[VBATCH], l3[VBATCH];
+#pragma unroll
+                for (int j = 0; j < VBATCH; ++j) {
+                    row[j] = -1;
+                    fl[j] = 0;
+                    e[j] = 0;
+                    if (b0 + j < cnt) {
+                        e[j] = mine[b0 + j];
+                        const uint8_t* ch = S.chunks + (size_t)(e[j] / SPCG_MAXREC) * SPCG_CHUNK_BYTES;
+                        const Rec R(ch + *(const uint16_t*)(ch + 8 + 2 * (e[j] % SPCG_MAXREC)));
+                        fl[j] = R.flags();
+                        row[j] = R.row(lane);
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < VBATCH; ++j) {      // every load of the batch before any use
+                    l0[j] = l1[j] = l2[j] = l3[j] = 0.0;
+                    if (row[j] >= 0) {
+                        if (!(fl[j] & REC_UPPER)) {
+                            if (kind == K_ITER) {
+                                l0[j] = __ldcg(P.r + row[j]);
+                                l1[j] = __ldcg(P.w + row[j]);
+                                l2[j] = __ldcg(P.x + row[j]);
+                                l3[j] = __ldcg(P.p + row[j]);
+                            } else {
+                                l0[j] = __ldcg(rin + row[j]);
+                            }
+                        } else {
+                            l0[j] = __ldcg(yin + row[j]);
+                            if (rdot) l1[j] = __ldcg(rdot + row[j]);
+                        }
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < VBATCH; ++j) {
+                    if (b0 + j >= cnt) continue;
+                    const int slot = e[j] / SPCG_MAXREC, r = e[j] % SPCG_MAXREC;
+                    if (row[j] >= 0) {
+                        double* vec = side_vec(S, slot, r);
+                        if (!(fl[j] & REC_UPPER)) {
+                            double ri = l0[j];
+                            if (kind == K_ITER) {
+                                ri = l0[j] - alpha * l1[j];
+                                P.r[row[j]] = ri;
+                                P.x[row[j]] = l2[j] + alpha * l3[j];
+                            } else if (kind == K_PRO) {
+                                if (rin != P.r) P.r[row[j]] = ri;
+                                if (!P.use_x0) P.x[row[j]] = 0.0;
+                            }
+                            rr = fma(ri, ri, rr);
+                            vec[lane] = ri;
+                        } else {
+                            vec[lane] = l0[j];
+                            side_aux(S, slot, r)[lane] = l1[j];
+                        }
+                    }
+                    if (lane == 0) *side_mask(S, slot, r) = 0u;
+                }
+            }
+            __syncwarp();
+            if (lane == 0)
+                for (int i = i0; i < i1; ++i) mbar_arrive(&S.vfull[(q0 + i) % SPCG_NCHUNK]);
+            i0 = i1;
         }
     } else if (warp >= POLLER_WARP && warp < POLLER_WARP + NPOLL) {
         const int pw = warp - POLLER_WARP;
@@ -1488,7 +1565,7 @@ extern "C" int spcg_dbg_counts(unsigned long long* out) {
         cudaMemcpyToSymbol(g_dbg_counts, &d, sizeof(d));
         return 0;
     }
-    cudaMemcpy(out, d, 24, cudaMemcpyDeviceToHost);
+    cudaMemcpy(out, d, 64, cudaMemcpyDeviceToHost);
     cudaMemset(d, 0, 64);
     return 1;
 }

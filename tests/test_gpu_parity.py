@@ -147,3 +147,15 @@ def test_tridiagonal_one_iteration():
         x, info = h.solve(_dev(b), eps=1e-12, kmax=50)
         assert info["iterations"] == 1, ex       # ILU(0) of a tridiagonal matrix is exact (P8)
         h.close()
+
+
+def test_calibrate_handoffs_are_ordered():
+    """Chain-floor calibration: every handoff measured, positive and
+    in the order the hardware fixes (intra-CTA < cross-CTA flag < grid barrier)."""
+    c = lib.calibrate(0)
+    assert c["sms"] >= 100
+    for k in ("grid_sync_ns", "graph_kernel_ns", "flag_same_die_ns", "flag_cross_die_ns", "syncthreads_ns",
+              "cluster_sync_ns"):
+        assert 0.0 < c[k] < 1e5, (k, c)
+    assert c["syncthreads_ns"] < c["flag_same_die_ns"] <= c["flag_cross_die_ns"]
+    assert c["flag_same_die_ns"] < c["grid_sync_ns"]
