@@ -321,10 +321,11 @@ def chain_floor(calib: dict, info: dict, bytes_per_iter: float, peak_gbs: float,
     lv = info["levels_L"] + info["levels_U"]
     per = {"grid_sync": calib["grid_sync_ns"], "graph_kernel": calib["graph_kernel_ns"],
            "flag_same_die": calib["flag_same_die_ns"], "flag_cross_die": calib["flag_cross_die_ns"],
+           "ll_flag_same_die": calib["flag_relaxed_same_die_ns"], "ll_flag_cross_die": calib["flag_relaxed_cross_die_ns"],
            "syncthreads": calib["syncthreads_ns"], "cluster_sync": calib["cluster_sync_ns"]}
     floors = {k: lv * v * 1e-3 for k, v in per.items()}              # us per iteration
-    own = {"level": "grid_sync", "syncfree": "flag_same_die", "chunked": "flag_same_die"}.get(
-        info["sptrsv_name"], "flag_same_die")
+    own = {"level": "grid_sync", "syncfree": "ll_flag_same_die", "chunked": "ll_flag_same_die"}.get(
+        info["sptrsv_name"], "ll_flag_same_die")
     hbm_us = bytes_per_iter / (peak_gbs * 1e9) * 1e6
     return {"levels": lv, "handoff_ns": per, "floor_us_per_iter": floors, "executor_handoff": own,
             "chain_floor_us_per_iter": floors[own], "hbm_floor_us_per_iter": hbm_us,

@@ -126,6 +126,8 @@ typedef struct {
     int64_t device_bytes;       /* device memory held by the handle */
     double algo_bytes_per_iter; /* B_iter: what one iteration must move */
     double algo_flops_per_iter;
+    int32_t partition;          /* CHUNKED: row partition the inspector chose — 0 contiguous, 1 strided,
+                                   2 affinity, 3 components; -1 otherwise */
 } spcg_setup_info_t;
 
 typedef struct {
@@ -214,6 +216,8 @@ typedef struct {
     double sm_clock_mhz;        /* cudaDevAttrClockRate */
     int32_t sms;
     int32_t flag_pairs_near;    /* CTA pairs classified as same-die (of sms - 1) */
+    double flag_relaxed_same_die_ns;   /* as flag_*, relaxed (volatile) accesses: the LL-flag handoff */
+    double flag_relaxed_cross_die_ns;
 } spcg_calib_t;
 spcg_status_t spcg_calibrate(int32_t device, spcg_calib_t* out);
 

@@ -75,7 +75,8 @@ class SetupInfo(ctypes.Structure):
                 ("setup_ms_symbolic", ctypes.c_double), ("setup_ms_numeric", ctypes.c_double),
                 ("setup_ms_layout", ctypes.c_double), ("setup_ms_upload", ctypes.c_double),
                 ("sptrsv", ctypes.c_int32), ("parts", ctypes.c_int32), ("device_bytes", ctypes.c_int64),
-                ("algo_bytes_per_iter", ctypes.c_double), ("algo_flops_per_iter", ctypes.c_double)]
+                ("algo_bytes_per_iter", ctypes.c_double), ("algo_flops_per_iter", ctypes.c_double),
+                ("partition", ctypes.c_int32)]
 
 
 class SolveInfo(ctypes.Structure):
@@ -136,7 +137,8 @@ class Calib(ctypes.Structure):
     _fields_ = [("grid_sync_ns", ctypes.c_double), ("graph_kernel_ns", ctypes.c_double),
                 ("flag_same_die_ns", ctypes.c_double), ("flag_cross_die_ns", ctypes.c_double),
                 ("syncthreads_ns", ctypes.c_double), ("cluster_sync_ns", ctypes.c_double),
-                ("sm_clock_mhz", ctypes.c_double), ("sms", ctypes.c_int32), ("flag_pairs_near", ctypes.c_int32)]
+                ("sm_clock_mhz", ctypes.c_double), ("sms", ctypes.c_int32), ("flag_pairs_near", ctypes.c_int32),
+                ("flag_relaxed_same_die_ns", ctypes.c_double), ("flag_relaxed_cross_die_ns", ctypes.c_double)]
 
 
 def calibrate(device: int = 0) -> dict:
@@ -207,6 +209,8 @@ class SPCG:
         self.info = {f[0]: (list(getattr(si, f[0])) if isinstance(getattr(si, f[0]), ctypes.Array)
                             else getattr(si, f[0])) for f in SetupInfo._fields_}
         self.info["sptrsv_name"] = SPTRSV_NAME.get(self.info["sptrsv"], "?")
+        self.info["partition_name"] = {0: "contiguous", 1: "strided", 2: "affinity", 3: "components"}.get(
+            self.info["partition"], "-")
 
     def close(self):
         h = getattr(self, "_h", None)

@@ -148,7 +148,16 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             sms = spcg_dev_sm_count(opt.device);
             if (sms <= 0) { delete h; return SPCG_ERR_CUDA; }
         }
-        int strategy = opt.sptrsv == SPCG_SPTRSV_AUTO ? SPCG_SPTRSV_CHUNKED : opt.sptrsv;
+        // AUTO: the chunked executor streams thread-per-row records of <= SPCG_WCAP entry
+        // columns; rows wider than that (ILU(K) fill of 3-D stencils: ~57 entries per L row
+        // for 27-point ILU(2)) need continuation records on the serial chain, where the
+        // level-scheduled executor (grid barrier per wavefront, the design of [36]) is faster
+        // (measured: FEM 48^3 ILU(2) 26 vs 31.5 ms per iteration).
+        int strategy = opt.sptrsv;
+        if (strategy == SPCG_SPTRSV_AUTO) {
+            const double wl = h->n > 0 ? (double)h->F.L.nnz() / (double)h->n : 0.0;
+            strategy = (h->identity || wl <= (double)SPCG_WCAP) ? SPCG_SPTRSV_CHUNKED : SPCG_SPTRSV_LEVEL;
+        }
         if (strategy < 1 || strategy > 3) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }
         int parts = opt.parts;
         if (parts <= 0) parts = h->n <= 16384 ? 1 : sms;
@@ -193,6 +202,11 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         I.sptrsv = strategy;
         I.parts = parts;
         I.device_bytes = bytes;
+        {
+            static const char* kinds[] = {"contiguous", "strided", "affinity", "components"};
+            I.partition = -1;
+            for (int k = 0; k < 4; ++k) if (h->lay.partition == kinds[k]) I.partition = k;
+        }
         // B_iter: 12 B per stored entry of A, L_s, U_s; 1/u_ii; three row
         // pointers; two level_rows arrays; 120 B of vector traffic per row.
         const double n = (double)h->n;

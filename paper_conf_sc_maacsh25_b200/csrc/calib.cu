@@ -61,7 +61,26 @@ __global__ void k_gridsync(unsigned* bar, int iters, unsigned long long* out) {
 // 2. empty kernel for the graph chain
 __global__ void k_empty() {}
 
-// 3. ping-pong between CTA 0 and CTA j, j = 1..G-1 in turn
+__device__ __forceinline__ unsigned ld_vol(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_vol(unsigned* p, unsigned v) {
+    asm volatile("st.volatile.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+template <bool RELAXED>
+__device__ __forceinline__ unsigned ld_flag(const unsigned* p) { return RELAXED ? ld_vol(p) : ld_acq(p); }
+template <bool RELAXED>
+__device__ __forceinline__ void st_flag(unsigned* p, unsigned v) {
+    if (RELAXED) st_vol(p, v);
+    else st_rel(p, v);
+}
+
+// 3. ping-pong between CTA 0 and CTA j, j = 1..G-1 in turn.  RELAXED: volatile
+// (relaxed) accesses with the value carrying its own validity, as the solver's
+// LL flags do; otherwise release store / acquire load.
+template <bool RELAXED>
 __global__ void k_pingpong(unsigned* ping, unsigned* pong, unsigned* turn, int rounds, unsigned long long* rt_ns,
                            int* smid) {
     const int j = blockIdx.x;
@@ -76,8 +95,8 @@ __global__ void k_pingpong(unsigned* ping, unsigned* pong, unsigned* turn, int r
             unsigned long long t0 = 0;
             for (int t = 1; t <= rounds + 8; ++t) {
                 if (t == 9) t0 = gtime();
-                st_rel(ping + p, (unsigned)t);
-                while (ld_acq(pong + p) != (unsigned)t) {
+                st_flag<RELAXED>(ping + p, (unsigned)t);
+                while (ld_flag<RELAXED>(pong + p) != (unsigned)t) {
                 }
             }
             rt_ns[p] = gtime() - t0;
@@ -86,9 +105,9 @@ __global__ void k_pingpong(unsigned* ping, unsigned* pong, unsigned* turn, int r
     } else {
         while (ld_acq(turn) != (unsigned)j) __nanosleep(256);
         for (int t = 1; t <= rounds + 8; ++t) {
-            while (ld_acq(ping + j) != (unsigned)t) {
+            while (ld_flag<RELAXED>(ping + j) != (unsigned)t) {
             }
-            st_rel(pong + j, (unsigned)t);
+            st_flag<RELAXED>(pong + j, (unsigned)t);
         }
     }
 }
@@ -184,7 +203,7 @@ extern "C" spcg_status_t spcg_calibrate(int32_t device, spcg_calib_t* out) {
         }
         out->graph_kernel_ns = (ms_b - ms_a) * 1e6 / 10.0 / 180.0;
     }
-    {   // 3. flag ping-pong CTA 0 <-> CTA j
+    for (int relaxed = 0; relaxed < 2; ++relaxed) {   // 3. flag ping-pong CTA 0 <-> CTA j
         int rounds = 200;
         unsigned* ping = dbuf + 4;
         unsigned* pong = dbuf + 4 + 1024;
@@ -192,7 +211,8 @@ extern "C" spcg_status_t spcg_calibrate(int32_t device, spcg_calib_t* out) {
         const int G = std::min(sms, 1024);
         CKC(cudaMemsetAsync(dbuf, 0, sizeof(unsigned) * (4 + 2 * 1024), s));
         void* args[] = {&ping, &pong, &turn, &rounds, &dres, &dsm};
-        CKC(cudaLaunchCooperativeKernel((void*)k_pingpong, dim3(G), dim3(32), args, 0, s));
+        CKC(cudaLaunchCooperativeKernel(relaxed ? (void*)k_pingpong<true> : (void*)k_pingpong<false>, dim3(G), dim3(32),
+                                        args, 0, s));
         rt.resize(G);
         smid.resize(G);
         CKC(cudaMemcpyAsync(rt.data(), dres, 8 * G, cudaMemcpyDeviceToHost, s));
@@ -208,9 +228,14 @@ extern "C" spcg_status_t spcg_calibrate(int32_t device, spcg_calib_t* out) {
         for (size_t i = ow.size() / 4; i + 1 < ow.size() * 3 / 4 + 1 && i + 1 < ow.size(); ++i)
             if (ow[i + 1] - ow[i] > best) { best = ow[i + 1] - ow[i]; cut = i + 1; }
         std::vector<double> near(ow.begin(), ow.begin() + cut), far(ow.begin() + cut, ow.end());
-        out->flag_same_die_ns = median(near);
-        out->flag_cross_die_ns = far.empty() ? median(near) : median(far);
-        out->flag_pairs_near = (int32_t)near.size();
+        if (relaxed) {
+            out->flag_relaxed_same_die_ns = median(near);
+            out->flag_relaxed_cross_die_ns = far.empty() ? median(near) : median(far);
+        } else {
+            out->flag_same_die_ns = median(near);
+            out->flag_cross_die_ns = far.empty() ? median(near) : median(far);
+            out->flag_pairs_near = (int32_t)near.size();
+        }
     }
     {   // 4a. __syncthreads
         int iters = 20000;

@@ -429,6 +429,14 @@ constexpr int VEC_WARP0 = POLLER_WARP + NPOLL;
 constexpr int NVEC = 4;
 constexpr int SOLVER_WARP0 = VEC_WARP0 + NVEC;
 static_assert(SOLVER_WARP0 + SPCG_NSOLVER == NWARP, "warp roles must fill the CTA");
+#ifndef SPCG_SOLVER_UNROLL
+#define SPCG_SOLVER_UNROLL 4       // record pairs per chunk unrolled in the solver (MAXREC / 2 = all)
+#endif
+#ifndef SPCG_PHASE_NOINLINE
+#define SPCG_PHASE_NOINLINE 0      // 1: one shared copy of the chunked phase (smaller code, but Params then
+                                   // live in local memory: 1.5x slower per iteration, measured)
+#endif
+constexpr int kSolverUnroll = SPCG_SOLVER_UNROLL;
 constexpr int POLL_AHEAD = 8;                     // records
 #ifndef SPCG_VGROUP
 #define SPCG_VGROUP 4
@@ -504,6 +512,15 @@ __device__ __forceinline__ bool mbar_wait(uint64_t* b, unsigned parity, Scal* sc
     return mbar_try(b, parity) || mbar_wait_slow(b, parity, sc);
 }
 __device__ __forceinline__ bool warp_ok(bool ok) { return __all_sync(0xffffffffu, ok); }
+// Poller -> solver handoff of a resolved external sum through shared memory:
+// the poller stores the value, fences (acq_rel, CTA scope: orders its two
+// shared-memory stores without waiting for the SM's outstanding global
+// stores, which membar.cta = fence.sc.cta would), then sets the mask bit; the
+// solver reads the mask and then the value with volatile loads (kept in program
+// order by the compiler; shared-memory accesses of one thread are performed
+// in order).  No fence on the solver's critical path.
+__device__ __forceinline__ void fence_acq_rel_cta() { asm volatile("fence.acq_rel.cta;" ::: "memory"); }
+__device__ __forceinline__ double lds_volatile(const double* p) { return *(const volatile double*)p; }
 // After an abort the ring may hold stale chunks: roles must stop parsing them.
 // Warp-collective code must take this decision warp-uniformly (a per-lane read
 // of a racy flag lets lanes disagree; a divergent break then deadlocks the
@@ -607,7 +624,7 @@ __device__ __forceinline__ bool ext_try(const Rec& R, int lane, int ne, const ui
     return ok;
 }
 
-__device__ double ext_wait(const Rec& R, int lane, int ne, const uint4* mb, unsigned ep, Scal* sc) {
+__device__ __noinline__ double ext_wait(const Rec& R, int lane, int ne, const uint4* mb, unsigned ep, Scal* sc) {
     double acc;
     if (ext_try(R, lane, ne, mb, ep, acc)) return acc;
     acc = 0.0;
@@ -736,14 +753,13 @@ __device__ __noinline__ double2 slow_record(const uint8_t* p, int fl, int wd, in
         double e = 0.0;
         if (row >= 0 && ne > 0) {
             const unsigned m = *(volatile unsigned*)(side_rec + 96);
-            if (m & (1u << lane)) { __threadfence_block(); e = side_rec[64 + lane]; }
+            if (m & (1u << lane)) e = lds_volatile(side_rec + 64 + lane);
             else e = ext_wait(R, lane, ne, mb, ep, sc);
         }
         acc = vec - e;
     } else {
         acc = acc_carry;
-        if (row >= 0)
-            for (int k = 0; k < ne; ++k) acc = fma(-R.val(k, lane), ll_wait(mb + (-R.src(k, lane) - 1), ep, sc), acc);
+        if (row >= 0 && ne > 0) acc -= ext_wait(R, lane, ne, mb, ep, sc);
     }
     if (row >= 0) acc = ring_terms_dispatch(wd, p, lane, ne, len, yring, acc);
     if ((fl & REC_LAST) && row >= 0) {
@@ -762,6 +778,9 @@ __device__ __noinline__ double2 slow_record(const uint8_t* p, int fl, int wd, in
     return make_double2(acc, rz);
 }
 
+#ifndef SPCG_DEBUG_COUNTS
+#define SPCG_DEBUG_COUNTS 0      // debug builds only (-DSPCG_DEBUG_COUNTS=1, tools/diag.py): no cost otherwise
+#endif
 __device__ unsigned long long* g_dbg_counts = nullptr;   // debug: [0] fast, [1] ext-fast, [2] slow
 template <bool UPPER, bool PRO>
 __device__ __forceinline__ void solve_record(const SolveCtx& C, const Prep& X, int slot, int lane, double& acc_carry,
@@ -782,10 +801,10 @@ __device__ __forceinline__ void solve_record(const SolveCtx& C, const Prep& X, i
         const unsigned m = *(volatile unsigned*)side_mask(*C.S, slot, X.r);
         const bool have = ne == 0 || (m >> lane) & 1u;
         const bool all_have = __all_sync(0xffffffffu, have);
-        if (g_dbg_counts && lane == 0) atomicAdd(g_dbg_counts + (all_have ? 1 : 2), 1ull);
+        if (SPCG_DEBUG_COUNTS && g_dbg_counts && lane == 0) atomicAdd(g_dbg_counts + (all_have ? 1 : 2), 1ull);
         if (all_have) {
             double e = 0.0;
-            if (ne > 0) { __threadfence_block(); e = side_ext(*C.S, slot, X.r)[lane]; }
+            if (ne > 0) e = lds_volatile(side_ext(*C.S, slot, X.r) + lane);
             double d[WP];
 #pragma unroll
             for (int k = 0; k < WP; ++k) d[k] = C.yring[X.sidx[k]];
@@ -802,7 +821,7 @@ __device__ __forceinline__ void solve_record(const SolveCtx& C, const Prep& X, i
             rz = o.y;
         }
     } else {
-        if (g_dbg_counts && lane == 0) atomicAdd(g_dbg_counts + 6, 1ull);
+        if (SPCG_DEBUG_COUNTS && g_dbg_counts && lane == 0) atomicAdd(g_dbg_counts + 6, 1ull);
         const double2 o = slow_record<UPPER, PRO>(X.p, X.fl, X.wd, X.row, X.meta, X.r, X.vec, X.aux, acc_carry, rz,
                                                   side_vec(*C.S, slot, X.r), C.yring, C.out, C.rdot, C.pvec, C.mb,
                                                   C.sc, C.ep, C.pb, C.mask);
@@ -821,7 +840,7 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
                                                long long recn, double& rz, const Params& P, long long kk) {
     const int lane = threadIdx.x & 31;
     double acc_carry = 0.0;
-    unsigned long long* dbg = g_dbg_counts;     // debug (SPCG_COUNT): solver wait / busy cycles
+    unsigned long long* dbg = SPCG_DEBUG_COUNTS ? g_dbg_counts : nullptr;   // debug: solver wait / busy cycles
     long long t_wait = 0, t_sec = dbg ? clock64() : 0;
     const long long recn0 = recn;
     for (int i = ib; i < ie; ++i) {
@@ -834,7 +853,7 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
         const int nrec = *(const uint16_t*)ch;
         Prep A, B;
         if (nrec > 0) prep_record<UPPER>(A, S, ch, slot, 0, lane);
-#pragma unroll
+#pragma unroll kSolverUnroll
         for (int r = 0; r < SPCG_MAXREC; r += 2) {
             if (r + 1 < nrec) prep_record<UPPER>(B, S, ch, slot, r + 1, lane);
             if (r < nrec) {
@@ -860,7 +879,12 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
 
 // One triangular-solve phase of a part: chunks [c0, c1) of its stream (L section,
 // U section or both).  All threads of the CTA call it.
-__device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st, int c0, int c1, int cu, int kind,
+#if SPCG_PHASE_NOINLINE
+__device__ __noinline__
+#else
+__device__ __forceinline__
+#endif
+void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st, int c0, int c1, int cu, int kind,
                               const double* rin, double* y, const double* yin, double* z, const double* rdot,
                               unsigned ep, double alpha, double& rr, double& rz, int64_t pb) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -1028,7 +1052,7 @@ __device__ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st
                         __syncwarp();
                         if (ok) {
                             side_ext(S, slot, r)[lane] = e;
-                            __threadfence_block();
+                            fence_acq_rel_cta();
                             atomicOr(side_mask(S, slot, r), 1u << lane);
                             need = false;
                         }

@@ -302,11 +302,63 @@ static void partition_contiguous(const Factors& F, int P, const std::vector<int3
     }
 }
 
+// Connected components of the dependency graph of L (undirected), packed onto
+// the parts largest first (LPT by rows).  When sparsification decouples the
+// matrix into independent blocks (the layered field: Algorithm 2 removes the
+// weak couplings across the low-conductivity columns) this
+// partition has no cross-CTA dependency at all: every wavefront chain stays in
+// one CTA's shared-memory ring.  Returns the number of components.
+static int64_t partition_components(const Factors& F, int P, Partition& out) {
+    const int64_t n = F.L.n;
+    std::vector<int32_t> par(n);
+    for (int64_t i = 0; i < n; ++i) par[i] = (int32_t)i;
+    auto find = [&](int32_t x) {
+        while (par[x] != x) { par[x] = par[par[x]]; x = par[x]; }
+        return x;
+    };
+    for (int64_t i = 0; i < n; ++i)
+        for (int64_t q = F.L.rp[i]; q < F.L.rp[i + 1]; ++q) {
+            const int32_t a = find((int32_t)i), b = find(F.L.col[q]);
+            if (a != b) par[std::max(a, b)] = std::min(a, b);
+        }
+    std::vector<int32_t> comp(n), size_of;
+    std::vector<int32_t> id(n, -1);
+    for (int64_t i = 0; i < n; ++i) {
+        const int32_t r = find((int32_t)i);
+        if (id[r] < 0) { id[r] = (int32_t)size_of.size(); size_of.push_back(0); }
+        comp[i] = id[r];
+        size_of[id[r]]++;
+    }
+    const int64_t nc = (int64_t)size_of.size();
+    std::vector<int32_t> order(nc);
+    for (int64_t c = 0; c < nc; ++c) order[c] = (int32_t)c;
+    std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return size_of[a] > size_of[b]; });
+    std::vector<int64_t> load(P, 0);
+    std::vector<int32_t> part_of_comp(nc, 0);
+    for (int32_t c : order) {
+        int best = 0;
+        for (int p = 1; p < P; ++p) if (load[p] < load[best]) best = p;
+        part_of_comp[c] = best;
+        load[best] += size_of[c];
+    }
+    out.parts = P;
+    out.part_of.assign(n, 0);
+    for (int64_t i = 0; i < n; ++i) out.part_of[i] = part_of_comp[comp[i]];
+    out.rows.assign(P, {});
+    out.lidx.assign(n, 0);
+    for (int64_t i = 0; i < n; ++i) {
+        const int p = out.part_of[i];
+        out.lidx[i] = (int32_t)out.rows[p].size();
+        out.rows[p].push_back((int32_t)i);
+    }
+    return nc;
+}
+
 // Executor model used to pick a partition: every part walks its wavefront groups
 // in order, a slice of <= 32 rows costs t_rec, and a dependency produced by
 // another part is usable H after it was produced.  Returns the modelled time of
 // one forward solve (the backward solve mirrors it).
-static double model_solve_time(const Factors& F, const Partition& PT, double t_rec, double H) {
+static double model_solve_time(const Factors& F, const Partition& PT, double t_rec, double t_ext, double H) {
     const int64_t n = F.L.n;
     std::vector<int64_t> lp(F.wL + 1, 0);
     for (int64_t i = 0; i < n; ++i) lp[F.levL[i] + 1]++;
@@ -318,6 +370,7 @@ static double model_solve_time(const Factors& F, const Partition& PT, double t_r
     }
     std::vector<double> fin(n, 0.0), clock(PT.parts, 0.0), ready(PT.parts, 0.0);
     std::vector<int32_t> cnt(PT.parts, 0), touched;
+    std::vector<char> ext(PT.parts, 0);
     for (int64_t l = 0; l < F.wL; ++l) {
         touched.clear();
         for (int64_t t = lp[l]; t < lp[l + 1]; ++t) {
@@ -326,12 +379,14 @@ static double model_solve_time(const Factors& F, const Partition& PT, double t_r
             if (cnt[p]++ == 0) { touched.push_back(p); ready[p] = clock[p]; }
             for (int64_t q = F.L.rp[i]; q < F.L.rp[i + 1]; ++q) {
                 const int32_t j = F.L.col[q];
-                if (PT.part_of[j] != p) ready[p] = std::max(ready[p], fin[j] + H);
+                if (PT.part_of[j] != p) { ready[p] = std::max(ready[p], fin[j] + H); ext[p] = 1; }
             }
         }
         for (int p : touched) {
-            clock[p] = ready[p] + t_rec * (double)((cnt[p] + 31) / 32);
+            // a record with cross-CTA terms costs more: poller handoff + flag reads
+            clock[p] = ready[p] + (ext[p] ? t_ext : t_rec) * (double)((cnt[p] + 31) / 32);
             cnt[p] = 0;
+            ext[p] = 0;
         }
         for (int64_t t = lp[l]; t < lp[l + 1]; ++t) fin[lrows[t]] = clock[PT.part_of[lrows[t]]];
     }
@@ -356,7 +411,9 @@ static int64_t dominant_stride(const Factors& F) {
 // Inspector: build candidate partitions and keep the one the model says is fastest.
 static void partition_rows(const Factors& F, int P, Partition& out, std::string* chosen) {
     const int64_t n = F.L.n;
-    const double T_REC = 0.45, H = 1.0;          // microseconds, measured on B200
+    // microseconds per record without / with cross-CTA terms, handoff latency: measured on
+    // B200 (tools/diag.py timelines)
+    const double T_REC = 0.45, T_EXT = 0.8, H = 1.0;
     std::vector<std::pair<std::string, Partition>> cand;
     std::vector<int32_t> ord(n);
     for (int64_t i = 0; i < n; ++i) ord[i] = (int32_t)i;
@@ -370,11 +427,15 @@ static void partition_rows(const Factors& F, int P, Partition& out, std::string*
         cand.push_back({"strided", std::move(p)});
     }
     { Partition p; partition_level_based(F, P, true, p); cand.push_back({"affinity", std::move(p)}); }
+    {
+        Partition p;
+        if (partition_components(F, P, p) >= P) cand.push_back({"components", std::move(p)});
+    }
     const char* force = getenv("SPCG_PART");
     double best = 1e300;
     size_t bi = 0;
     for (size_t c = 0; c < cand.size(); ++c) {
-        const double t = model_solve_time(F, cand[c].second, T_REC, H);
+        const double t = model_solve_time(F, cand[c].second, T_REC, T_EXT, H);
         if (getenv("SPCG_PART_VERBOSE")) fprintf(stderr, "[spcg] partition %s: modelled forward solve %.1f us\n", cand[c].first.c_str(), t);
         if (force ? cand[c].first == force : t < best) { best = force ? 0.0 : t; bi = c; }
     }

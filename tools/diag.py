@@ -19,6 +19,12 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import gen  # noqa: E402
+from paper_conf_sc_maacsh25_b200 import _build  # noqa: E402
+
+DBG_LIB = _build.LIB.replace("libspcg.so", "libspcg_dbg.so")
+if not os.path.exists(DBG_LIB):
+    _build.build(defines=["-DSPCG_DEBUG_COUNTS=1"], out=DBG_LIB)
+os.environ["SPCG_LIB"] = DBG_LIB
 import paper_conf_sc_maacsh25_b200 as spcg  # noqa: E402
 
 ap = argparse.ArgumentParser()
@@ -51,7 +57,7 @@ rel = (cta - t0) / 1e3                               # us
 iters = a.k
 out = {"n": A.n, "levels": [h.info["levels_L"], h.info["levels_U"]], "parts": parts,
        "ms_per_iter": si["iter_phase_ms"] / iters,
-       "counts": {"fast": int(cnt[0]), "ext_fast": int(cnt[1]), "ext_slow": int(cnt[2]), "other_slow": int(cnt[6]),
+       "partition": h.info.get("partition_name"), "counts": {"fast": int(cnt[0]), "ext_fast": int(cnt[1]), "ext_slow": int(cnt[2]), "other_slow": int(cnt[6]),
                   "records": int(cnt[5])},
        "solver_wait_frac": float(cnt[3]) / max(float(cnt[4]), 1.0),
        "solver_cycles_per_record": float(cnt[4]) / max(float(cnt[5]), 1.0) / parts * parts,

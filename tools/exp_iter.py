@@ -43,6 +43,6 @@ for mode in a.modes.split(","):
         ms.append(sf["iter_phase_ms"])
     out[mode] = {"k_conv": k_conv, "conv_ms": si["iter_phase_ms"], "ms_per_iter_forced": float(np.median(ms)) / a.k,
                  "levels": [h.info["levels_L"], h.info["levels_U"]], "sptrsv": h.info["sptrsv_name"],
-                 "partition": h.info.get("partition", "")}
+                 "partition": h.info.get("partition_name", "")}
     h.close()
 print(json.dumps(out))
