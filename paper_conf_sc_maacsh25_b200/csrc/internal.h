@@ -70,6 +70,16 @@ struct TriLayout {
     std::vector<int32_t> part_gptr;// [parts+1]  group ranges per part (chunked); levels: [0, ngroups]
     int32_t ngroups = 0;
     int64_t total_cols = 0;        // sum of slice widths
+    // LEVEL with wide rows (mean dependencies per row > SPCG_WCAP, e.g. ILU(K) fill):
+    // warp-per-row CSR in execution order (level, ascending row), read coalesced by
+    // the 32 lanes of a warp and reduced with shuffles.
+    bool wide = false;
+    std::vector<int32_t> wrow;     // [n] row at each position
+    std::vector<int64_t> wptr;     // [n+1] dependency range of each position
+    std::vector<int32_t> wcol;     // dependencies (U: diagonal excluded)
+    std::vector<double> wval;
+    std::vector<double> wdinv;     // [n] 1/u_ii per position (upper only)
+    std::vector<int32_t> wgptr;    // [ngroups+1] position range of each level
 };
 
 struct SpmvLayout {                // SELL-32 of the original A, natural row order

@@ -56,6 +56,13 @@ struct DevTri {
     const double* dinv;
     const int32_t* gptr;
     const int32_t* part_gptr;
+    int32_t wide;                  // LEVEL, wide rows: warp-per-row CSR below (layout.cpp)
+    const int32_t* wrow;
+    const int64_t* wptr;
+    const int32_t* wcol;
+    const double* wval;
+    const double* wdinv;
+    const int32_t* wgptr;
 };
 
 struct DevA {
@@ -391,12 +398,107 @@ __device__ __forceinline__ void tri_slice(const Params& P, const DevTri& T, int6
     __syncwarp();
 }
 
+// LEVEL executor, wide rows (ILU(K) fill): one warp per row of the wavefront, the
+// lanes stride the row's dependencies (coalesced CSR reads, 2 entries per lane
+// prefetched before the previous wavefront's barrier completes), a fixed-order
+// shuffle reduction, lane 0 finishes the row (fused x/r update and ||r||^2 for L;
+// 1/u_ii, (r,z) and p0 for U).
+constexpr int WPF = 2;                 // entries per lane prefetched across the barrier
+template <bool UPPER>
+__device__ void tri_level_wide(const Params& P, const DevTri& T, int kind, const double* in, double* out,
+                               const double* rdot, double alpha, double& acc_dot, unsigned& gen) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t W = (int64_t)gridDim.x * NWARP;
+    const int64_t gw = (int64_t)blockIdx.x * NWARP + warp;
+    // prefetch state for the first position of this warp in level g
+    int64_t q = -1, e0 = 0, e1 = 0;
+    int row = -1;
+    int cpf[WPF];
+    double vpf[WPF];
+    auto prefetch = [&](int g) {
+        const int64_t p0 = __ldg(T.wgptr + g), p1 = __ldg(T.wgptr + g + 1);
+        q = p0 + gw < p1 ? p0 + gw : -1;
+        if (q >= 0) {
+            row = __ldg(T.wrow + q);
+            e0 = __ldg(T.wptr + q);
+            e1 = __ldg(T.wptr + q + 1);
+#pragma unroll
+            for (int u = 0; u < WPF; ++u) {
+                const int64_t e = e0 + lane + 32 * u;
+                cpf[u] = e < e1 ? __ldg(T.wcol + e) : -1;
+                vpf[u] = e < e1 ? __ldg(T.wval + e) : 0.0;
+            }
+        }
+    };
+    if (T.ngroups > 0) prefetch(0);
+    for (int g = 0; g < T.ngroups; ++g) {
+        const int64_t p1 = __ldg(T.wgptr + g + 1);
+        bool first = true;
+        for (; q >= 0 && q < p1; q += W) {
+            if (!first) {
+                row = __ldg(T.wrow + q);
+                e0 = __ldg(T.wptr + q);
+                e1 = __ldg(T.wptr + q + 1);
+#pragma unroll
+                for (int u = 0; u < WPF; ++u) {
+                    const int64_t e = e0 + lane + 32 * u;
+                    cpf[u] = e < e1 ? __ldg(T.wcol + e) : -1;
+                    vpf[u] = e < e1 ? __ldg(T.wval + e) : 0.0;
+                }
+            }
+            first = false;
+            // the row's own operands first (independent of the gathers)
+            double r0 = 0.0, w0 = 0.0, x0 = 0.0, p0v = 0.0, a0 = 0.0;
+            if (lane == 0) {
+                if (!UPPER) {
+                    if (kind == K_ITER) { r0 = __ldcg(P.r + row); w0 = __ldcg(P.w + row); x0 = __ldcg(P.x + row); p0v = __ldcg(P.p + row); }
+                    else r0 = __ldcg(in + row);
+                } else {
+                    r0 = __ldcg(in + row);
+                    if (rdot) a0 = __ldcg(rdot + row);
+                }
+            }
+            double part = 0.0;
+#pragma unroll
+            for (int u = 0; u < WPF; ++u)
+                if (cpf[u] >= 0) part = fma(vpf[u], __ldcg(out + cpf[u]), part);
+            for (int64_t e = e0 + lane + 32 * WPF; e < e1; e += 32) part = fma(__ldg(T.wval + e), __ldcg(out + __ldg(T.wcol + e)), part);
+            part = warp_sum(part);
+            if (lane == 0) {
+                double acc;
+                if (!UPPER) {
+                    double ri = r0;
+                    if (kind == K_ITER) {
+                        ri = r0 - alpha * w0;
+                        P.r[row] = ri;
+                        P.x[row] = x0 + alpha * p0v;
+                    } else if (kind == K_PRO) {
+                        if (in != P.r) P.r[row] = ri;
+                        if (!P.use_x0) P.x[row] = 0.0;
+                    }
+                    acc_dot = fma(ri, ri, acc_dot);
+                    acc = ri - part;
+                } else {
+                    acc = (r0 - part) * __ldg(T.wdinv + q);
+                    if (rdot) acc_dot = fma(a0, acc, acc_dot);
+                    if (kind == K_PRO) P.p[row] = acc;
+                }
+                out[row] = acc;
+            }
+        }
+        if (g + 1 < T.ngroups) prefetch(g + 1);     // independent of the barrier
+        grid_sync(P.sc, gen);
+    }
+}
+
 template <int STRAT, bool UPPER>
 __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const double* in, double* out,
                           const double* rdot, uint4* mb, unsigned ep, double alpha, double& acc_dot,
                           double* ring, unsigned& gen) {
     const int warp = threadIdx.x >> 5;
-    if (STRAT == ST_LEVEL) {
+    if (STRAT == ST_LEVEL && T.wide) {
+        tri_level_wide<UPPER>(P, T, kind, in, out, rdot, alpha, acc_dot, gen);
+    } else if (STRAT == ST_LEVEL) {
         const int64_t W = (int64_t)gridDim.x * NWARP;
         const int64_t gw = (int64_t)blockIdx.x * NWARP + warp;
         for (int g = 0; g < T.ngroups; ++g) {
@@ -1348,6 +1450,13 @@ static spcg_status_t upload_tri(spcg_device_t* d, const spcg::TriLayout& T, DevT
     if ((s = upload(d, T.dinv, &D.dinv))) return s;
     if ((s = upload(d, T.gptr, &D.gptr))) return s;
     if ((s = upload(d, T.part_gptr, &D.part_gptr))) return s;
+    D.wide = T.wide ? 1 : 0;
+    if ((s = upload(d, T.wrow, &D.wrow))) return s;
+    if ((s = upload(d, T.wptr, &D.wptr))) return s;
+    if ((s = upload(d, T.wcol, &D.wcol))) return s;
+    if ((s = upload(d, T.wval, &D.wval))) return s;
+    if ((s = upload(d, T.wdinv, &D.wdinv))) return s;
+    if ((s = upload(d, T.wgptr, &D.wgptr))) return s;
     return SPCG_OK;
 }
 

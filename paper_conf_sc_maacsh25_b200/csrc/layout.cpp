@@ -99,6 +99,31 @@ static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev,
     T.ngroups = (int32_t)grp_rows_ptr.size() - 1;
     (void)w;
 
+    // LEVEL + wide rows: warp-per-row CSR in execution order
+    {
+        int64_t deps = 0;
+        for (int64_t i = 0; i < n; ++i) deps += dep_end(i) - dep_begin(i);
+        T.wide = strategy == SPCG_SPTRSV_LEVEL && n > 0 && (double)deps / (double)n > (double)SPCG_WCAP;
+        if (T.wide) {
+            T.wrow.assign(order.begin(), order.end());
+            T.wgptr.assign(grp_rows_ptr.begin(), grp_rows_ptr.end());
+            T.wptr.assign(n + 1, 0);
+            for (int64_t t = 0; t < n; ++t) T.wptr[t + 1] = T.wptr[t] + (dep_end(order[t]) - dep_begin(order[t]));
+            T.wcol.resize(T.wptr[n]);
+            T.wval.resize(T.wptr[n]);
+            if (upper) T.wdinv.resize(n);
+            for (int64_t t = 0; t < n; ++t) {
+                const int32_t r = order[t];
+                int64_t e = T.wptr[t];
+                for (int64_t q = dep_begin(r); q < dep_end(r); ++q, ++e) {
+                    T.wcol[e] = M.col[q];
+                    T.wval[e] = M.val[q];
+                }
+                if (upper) T.wdinv[t] = 1.0 / M.val[M.rp[r]];
+            }
+        }
+    }
+
     // slices of <= 32 rows inside each group
     T.gptr.assign(1, 0);
     std::vector<int32_t> slice_start;    // index into order
