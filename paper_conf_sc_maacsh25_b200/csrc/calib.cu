@@ -34,24 +34,18 @@ __device__ __forceinline__ void st_rel(unsigned* p, unsigned v) {
     asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// 1. grid barrier (arrive counter + generation, the scheme of the solver kernel)
+// 1. grid barrier: the solver's scheme (monotonic arrival counter, release
+//    reduction, acquire spin until gen x gridDim)
 __global__ void k_gridsync(unsigned* bar, int iters, unsigned long long* out) {
-    unsigned gen = 0;
-    if (threadIdx.x == 0) gen = ld_acq(bar + 1);
     __syncthreads();
     const unsigned long long t0 = gtime();
     for (int it = 0; it < iters; ++it) {
         __syncthreads();
         if (threadIdx.x == 0) {
-            const unsigned g = gen;
-            if (atomicAdd(bar, 1u) == gridDim.x - 1) {
-                bar[0] = 0;
-                st_rel(bar + 1, g + 1);
-            } else {
-                while (ld_acq(bar + 1) == g) {
-                }
+            const unsigned target = (unsigned)(it + 1) * gridDim.x;
+            asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(bar), "r"(1u) : "memory");
+            while ((int)(ld_acq(bar) - target) < 0) {
             }
-            gen = g + 1;
         }
         __syncthreads();
     }
@@ -177,6 +171,7 @@ extern "C" spcg_status_t spcg_calibrate(int32_t device, spcg_calib_t* out) {
         int iters = 4000;
         void* args[] = {&dbuf, &iters, &dres};
         CKC(cudaLaunchCooperativeKernel((void*)k_gridsync, dim3(sms), dim3(256), args, 0, s));   // warm-up
+        CKC(cudaMemsetAsync(dbuf, 0, sizeof(unsigned) * 4, s));
         CKC(cudaLaunchCooperativeKernel((void*)k_gridsync, dim3(sms), dim3(256), args, 0, s));
         unsigned long long ns = 0;
         CKC(cudaMemcpyAsync(&ns, dres, 8, cudaMemcpyDeviceToHost, s));

@@ -208,27 +208,27 @@ __device__ __forceinline__ double ll_wait(const uint4* p, unsigned ep, Scal* sc)
     return ll_wait_slow(p, ep, sc);
 }
 
-// grid-wide barrier (all CTAs co-resident: cooperative launch)
+// grid-wide barrier (all CTAs co-resident: cooperative launch).  Monotonic
+// arrival counter (zeroed per launch with the Scal block): CTA thread 0 adds 1
+// with a release reduction (no round trip) and spins with acquire loads until
+// the counter reaches gen x gridDim — one L2 hop less than counter + reset +
+// generation flag (calibrated by spcg_calibrate, grid_sync_ns).
+__device__ __forceinline__ void red_release_add(unsigned* p, unsigned v) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 __device__ __forceinline__ void grid_sync(Scal* sc, unsigned& gen) {
     __syncthreads();
     if (gridDim.x > 1) {
         if (threadIdx.x == 0) {
-            unsigned g = gen;
-            __threadfence();
-            unsigned prev = atomicAdd(&sc->bar_count, 1u);
-            if (prev == gridDim.x - 1) {
-                atomicExch(&sc->bar_count, 0u);
-                __threadfence();
-                st_release_u32(&sc->bar_gen, g + 1);
-            } else {
-                const long long t0 = clock64();
-                while (ld_acquire_u32(&sc->bar_gen) == g) {
-                    if (ld_volatile_int(&sc->abort)) break;
-                    if (clock64() - t0 > SPIN_TIMEOUT_CYC) { atomicExch(&sc->abort, 1); break; }
-                }
+            const unsigned target = (gen + 1) * gridDim.x;
+            red_release_add(&sc->bar_count, 1u);
+            const long long t0 = clock64();
+            while ((int)(ld_acquire_u32(&sc->bar_count) - target) < 0) {
+                if (ld_volatile_int(&sc->abort)) break;
+                if (clock64() - t0 > SPIN_TIMEOUT_CYC) { atomicExch(&sc->abort, 1); break; }
             }
-            gen = g + 1;
         }
+        ++gen;
         __syncthreads();
     }
 }
@@ -415,6 +415,21 @@ __device__ void tri_level_wide(const Params& P, const DevTri& T, int kind, const
     int row = -1;
     int cpf[WPF];
     double vpf[WPF];
+    double r0 = 0.0, w0 = 0.0, x0 = 0.0, p0v = 0.0, a0 = 0.0, dv = 1.0;
+    // the row's own operands (lane 0): none of them is written by this solve's
+    // wavefronts, so they are loaded before the barrier that precedes their use
+    auto own = [&]() {
+        if (lane == 0) {
+            if (!UPPER) {
+                if (kind == K_ITER) { r0 = __ldcg(P.r + row); w0 = __ldcg(P.w + row); x0 = __ldcg(P.x + row); p0v = __ldcg(P.p + row); }
+                else r0 = __ldcg(in + row);
+            } else {
+                r0 = __ldcg(in + row);
+                if (rdot) a0 = __ldcg(rdot + row);
+                dv = __ldg(T.wdinv + q);
+            }
+        }
+    };
     auto prefetch = [&](int g) {
         const int64_t p0 = __ldg(T.wgptr + g), p1 = __ldg(T.wgptr + g + 1);
         q = p0 + gw < p1 ? p0 + gw : -1;
@@ -428,6 +443,7 @@ __device__ void tri_level_wide(const Params& P, const DevTri& T, int kind, const
                 cpf[u] = e < e1 ? __ldg(T.wcol + e) : -1;
                 vpf[u] = e < e1 ? __ldg(T.wval + e) : 0.0;
             }
+            own();
         }
     };
     if (T.ngroups > 0) prefetch(0);
@@ -445,19 +461,9 @@ __device__ void tri_level_wide(const Params& P, const DevTri& T, int kind, const
                     cpf[u] = e < e1 ? __ldg(T.wcol + e) : -1;
                     vpf[u] = e < e1 ? __ldg(T.wval + e) : 0.0;
                 }
+                own();
             }
             first = false;
-            // the row's own operands first (independent of the gathers)
-            double r0 = 0.0, w0 = 0.0, x0 = 0.0, p0v = 0.0, a0 = 0.0;
-            if (lane == 0) {
-                if (!UPPER) {
-                    if (kind == K_ITER) { r0 = __ldcg(P.r + row); w0 = __ldcg(P.w + row); x0 = __ldcg(P.x + row); p0v = __ldcg(P.p + row); }
-                    else r0 = __ldcg(in + row);
-                } else {
-                    r0 = __ldcg(in + row);
-                    if (rdot) a0 = __ldcg(rdot + row);
-                }
-            }
             double part = 0.0;
 #pragma unroll
             for (int u = 0; u < WPF; ++u)
@@ -479,7 +485,7 @@ __device__ void tri_level_wide(const Params& P, const DevTri& T, int kind, const
                     acc_dot = fma(ri, ri, acc_dot);
                     acc = ri - part;
                 } else {
-                    acc = (r0 - part) * __ldg(T.wdinv + q);
+                    acc = (r0 - part) * dv;
                     if (rdot) acc_dot = fma(a0, acc, acc_dot);
                     if (kind == K_PRO) P.p[row] = acc;
                 }
