@@ -949,7 +949,7 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
     const int lane = threadIdx.x & 31;
     double acc_carry = 0.0;
     unsigned long long* dbg = SPCG_DEBUG_COUNTS ? g_dbg_counts : nullptr;   // debug: solver wait / busy cycles
-    long long t_wait = 0, t_sec = dbg ? clock64() : 0;
+    long long t_wait = 0, t_sec = dbg ? clock64() : 0, t_prep = 0, t_solve = 0, nchunks = 0;
     const long long recn0 = recn;
     for (int i = ib; i < ie; ++i) {
         const unsigned q = q0 + i;
@@ -963,18 +963,24 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
         if (nrec > 0) prep_record<UPPER>(A, S, ch, slot, 0, lane);
 #pragma unroll kSolverUnroll
         for (int r = 0; r < SPCG_MAXREC; r += 2) {
+            long long tp = dbg ? clock64() : 0;
             if (r + 1 < nrec) prep_record<UPPER>(B, S, ch, slot, r + 1, lane);
+            if (dbg) { t_prep += clock64() - tp; tp = clock64(); }
             if (r < nrec) {
                 if (lane == 0) S.progress[0] = recn + r;
                 solve_record<UPPER, PRO>(C, A, slot, lane, acc_carry, rz);
             }
+            if (dbg) { t_solve += clock64() - tp; tp = clock64(); }
             if (r + 2 < nrec) prep_record<UPPER>(A, S, ch, slot, r + 2, lane);
+            if (dbg) { t_prep += clock64() - tp; tp = clock64(); }
             if (r + 1 < nrec) {
                 if (lane == 0) S.progress[0] = recn + r + 1;
                 solve_record<UPPER, PRO>(C, B, slot, lane, acc_carry, rz);
             }
+            if (dbg) t_solve += clock64() - tp;
         }
         recn += nrec;
+        ++nchunks;
         __syncwarp();
         if (lane == 0) mbar_arrive(&S.empty[slot]);
     }
@@ -982,6 +988,9 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
         atomicAdd(dbg + 3, (unsigned long long)t_wait);
         atomicAdd(dbg + 4, (unsigned long long)(clock64() - t_sec));
         atomicAdd(dbg + 5, (unsigned long long)(recn - recn0));
+        atomicAdd(dbg + 7, (unsigned long long)nchunks);
+        atomicAdd(dbg + 8, (unsigned long long)t_prep);
+        atomicAdd(dbg + 9, (unsigned long long)t_solve);
     }
 }
 
@@ -1699,12 +1708,12 @@ spcg_status_t spcg_dev_copy(spcg_device_t* d, void* dst, const void* src, size_t
 extern "C" int spcg_dbg_counts(unsigned long long* out) {
     static unsigned long long* d = nullptr;
     if (!d) {
-        if (cudaMalloc(&d, 64) != cudaSuccess) return -1;
-        cudaMemset(d, 0, 64);
+        if (cudaMalloc(&d, 128) != cudaSuccess) return -1;
+        cudaMemset(d, 0, 128);
         cudaMemcpyToSymbol(g_dbg_counts, &d, sizeof(d));
         return 0;
     }
-    cudaMemcpy(out, d, 64, cudaMemcpyDeviceToHost);
-    cudaMemset(d, 0, 64);
+    cudaMemcpy(out, d, 128, cudaMemcpyDeviceToHost);
+    cudaMemset(d, 0, 128);
     return 1;
 }

@@ -22,7 +22,7 @@ import gen  # noqa: E402
 from paper_conf_sc_maacsh25_b200 import _build  # noqa: E402
 
 DBG_LIB = _build.LIB.replace("libspcg.so", "libspcg_dbg.so")
-if not os.path.exists(DBG_LIB):
+if True:   # always rebuild: the knob is compile-time
     _build.build(defines=["-DSPCG_DEBUG_COUNTS=1"], out=DBG_LIB)
 os.environ["SPCG_LIB"] = DBG_LIB
 import paper_conf_sc_maacsh25_b200 as spcg  # noqa: E402
@@ -36,7 +36,7 @@ ap.add_argument("--mode", default="alg2")
 ap.add_argument("--sptrsv", default="chunked")
 a = ap.parse_args()
 
-lib = spcg.load()
+lib = spcg.load(DBG_LIB)
 lib.spcg_dbg_counts.argtypes = [ctypes.c_void_p]
 A = gen.make(a.family, *a.params)
 b, _ = gen.rhs(A)
@@ -44,7 +44,7 @@ bd = torch.from_numpy(b).cuda()
 h = spcg.SPCG(A, mode=a.mode, K=a.K, sptrsv=a.sptrsv, device=0)
 h.solve(bd, eps=0.0, kmax=a.k)                       # warm-up
 open(tr_path, "w").close()
-cnt = np.zeros(8, np.uint64)
+cnt = np.zeros(16, np.uint64)
 lib.spcg_dbg_counts(cnt.ctypes.data)                 # enable + zero
 _, si = h.solve(bd, eps=0.0, kmax=a.k)
 lib.spcg_dbg_counts(cnt.ctypes.data)
@@ -60,6 +60,11 @@ out = {"n": A.n, "levels": [h.info["levels_L"], h.info["levels_U"]], "parts": pa
        "partition": h.info.get("partition_name"), "counts": {"fast": int(cnt[0]), "ext_fast": int(cnt[1]), "ext_slow": int(cnt[2]), "other_slow": int(cnt[6]),
                   "records": int(cnt[5])},
        "solver_wait_frac": float(cnt[3]) / max(float(cnt[4]), 1.0),
+       "records_per_chunk": float(cnt[5]) / max(float(cnt[7]), 1.0),
+       "cycles_per_record": {"total": float(cnt[4]) / max(float(cnt[5]), 1.0),
+                             "vfull_wait": float(cnt[3]) / max(float(cnt[5]), 1.0),
+                             "prep": float(cnt[8]) / max(float(cnt[5]), 1.0),
+                             "solve": float(cnt[9]) / max(float(cnt[5]), 1.0)},
        "solver_cycles_per_record": float(cnt[4]) / max(float(cnt[5]), 1.0) / parts * parts,
        "timeline_us": {
            "L_first_record": [float(rel[:, 0].min()), float(np.median(rel[:, 0])), float(rel[:, 0].max())],
