@@ -97,11 +97,17 @@ def setup_rank(systems, device: int, mode: str = "alg2", **kw):
     return handles
 
 
-def solve_rank(handles, eps: float = 1e-8, kmax: int = 20000):
-    """Solve this rank's systems on its GPU; returns per-system results."""
+def solve_rank(handles, eps: float = 1e-8, kmax: int = 20000, host: bool = False):
+    """Solve this rank's systems on its GPU; returns per-system results.
+    host=True: the public host-pointer path (H2D of b and D2H of x inside each call)."""
     import torch
     out = []
     for s, A, b, h, st in handles:
+        if host:
+            xh, info = h.solve_host(b, eps=eps, kmax=kmax)
+            out.append(Result(s.index, s.family, A.n, info["iterations"], info["iter_phase_ms"], info["rnorm"],
+                              info["status"], h.info["chosen_pct"], h.info["levels_L"], float(np.sum(xh)), st))
+            continue
         bd = torch.from_numpy(b).to(f"cuda:{h.device}")
         x, info = h.solve(bd, eps=eps, kmax=kmax)
         out.append(Result(s.index, s.family, A.n, info["iterations"], info["iter_phase_ms"], info["rnorm"],
