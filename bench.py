@@ -173,6 +173,8 @@ def main():
     ap.add_argument("--parts", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--batch-count", type=int, default=64)
+    ap.add_argument("--sweep", default=None,
+                    help="comma list of fixed drop ratios t%% timed beside Alg. 2 and PCG (default: 1,5,10 for C4)")
     args = ap.parse_args()
     ws, rank, local = _dist()
     name = args.workload
@@ -254,6 +256,24 @@ def main():
                                  e2e=float(np.mean(e2e)), info=h.info)
     clocks = clk.summary()
     calib = spcg.calibrate(dev)
+    # C4 sparsification sweep, fixed t beside Alg. 2's choice and PCG (t = 0)
+    sweep_spec = args.sweep if args.sweep is not None else ("1,5,10" if name == "C4" else "")
+    sweep = []
+    for t in [float(v) for v in sweep_spec.split(",") if v.strip()]:
+        hs = spcg.SPCG(A, mode="fixed", fixed_pct=t, K=K, sptrsv=args.sptrsv, parts=args.parts, device=dev,
+                       stream=stream)
+        hs.solve(bd, xd, EPS, KMAX)
+        tms, tk = [], 0
+        for _ in range(max(1, min(args.steps, 3))):
+            flush.zero_()
+            _, inf = hs.solve(bd, xd, EPS, KMAX)
+            tms.append(inf["iter_phase_ms"])
+            tk = inf["iterations"]
+        sweep.append({"t_pct": t, "ms": float(np.mean(tms)), "iterations": tk, "ms_per_iter": float(np.mean(tms)) / max(tk, 1),
+                      "levels_L": hs.info["levels_L"], "m_t": hs.info["m_t"], "status": inf["status"],
+                      "partition": hs.info["partition_name"],
+                      "hbm_gbs_per_iter": hs.info["algo_bytes_per_iter"] * tk / (float(np.mean(tms)) * 1e-3) / 1e9})
+        hs.close()
 
     def mx(v):
         if ws == 1:
@@ -287,7 +307,7 @@ def main():
         "dtype": "f64", "data": "synthetic",
         "config": {"workload": WORKLOADS[name], "n": A.n, "nnz": A.nnz, "K": K, "eps": EPS,
                    "drop": "Algorithm 2 (tau=1, omega=10%, ratios 10/5/1)", "chosen_pct": si["chosen_pct"],
-                   "sptrsv": si["sptrsv_name"], "ctas": si["parts"],
+                   "sptrsv": si["sptrsv_name"], "ctas": si["parts"], "partition": si["partition_name"],
                    "l2": "flushed between steps (256 MiB write); timed region = the solve kernel only",
                    "replicas": ws},
         "iterations": s["k"], "ms_per_iter": s_ms / max(s["k"], 1),
@@ -295,6 +315,7 @@ def main():
         "levels": {"L": si["levels_L"], "U": si["levels_U"], "w_A": si["w_A"], "w_Ahat": si["w_Ahat"]},
         "pcg": {"value": p_ms, "iterations": p["k"], "ms_per_iter": p_ms / max(p["k"], 1), "hbm_gbs_per_iter": p_gbs,
                 "algo_bytes_per_iter": p_bi, "levels": {"L": pi["levels_L"], "U": pi["levels_U"]}},
+        "sweep": sweep or None,
         "spcg_vs_pcg": {"iter_phase_speedup": p_ms / s_ms,
                         "per_iter_speedup": (p_ms / max(p["k"], 1)) / (s_ms / max(s["k"], 1))},
         "paper_context": PAPER_CONTEXT,

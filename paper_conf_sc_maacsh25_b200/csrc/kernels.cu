@@ -38,6 +38,9 @@ using namespace spcg;
 namespace {
 
 constexpr int BLOCK = 256;
+#ifndef SPCG_CTAS_PER_SM
+#define SPCG_CTAS_PER_SM 1        // persistent CTAs per SM (2: two independent chains per SM, <= 128 registers)
+#endif
 constexpr int NWARP = BLOCK / 32;
 constexpr long long SPIN_TIMEOUT_CYC = 8ll * 1000 * 1000 * 1000;            // ~4 s of SM cycles: abort, never hang
 
@@ -1284,7 +1287,7 @@ __device__ void tri_solve(const Params& P, int sec, int kind, const double* rin,
 }
 
 template <int STRAT>
-__global__ void __launch_bounds__(BLOCK, 1) spcg_pcg_kernel(Params P) {
+__global__ void __launch_bounds__(BLOCK, SPCG_CTAS_PER_SM) spcg_pcg_kernel(Params P) {
     extern __shared__ __align__(128) double dyn[];
     double* ring = dyn;
     unsigned gen = 0;
