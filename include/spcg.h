@@ -183,6 +183,19 @@ spcg_status_t spcg_get_setup_info(spcg_handle_t h, spcg_setup_info_t* info);
 spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps, int64_t kmax,
                          uint32_t flags, spcg_solve_info_t* info);
 
+/* Asynchronous form of spcg_solve for running independent systems concurrently
+ * (the C5 batch): enqueues Algorithm 1 on the handle's stream
+ * and returns; b, x must be device pointers (SPCG_HOST_PTRS -> INVALID_ARG) and
+ * stay valid until spcg_solve_wait(h, info) has returned, which synchronises
+ * the stream and fills info exactly as spcg_solve does.  One solve in flight per
+ * handle (a second spcg_solve_async before the wait -> INVALID_ARG).  Handles
+ * set up on different streams run concurrently; each launch is cooperative, so
+ * the caller keeps the CTAs (setup opt.parts) of the solves in flight on one
+ * device within its SM count. */
+spcg_status_t spcg_solve_async(spcg_handle_t h, const double* b, double* x, double eps, int64_t kmax,
+                               uint32_t flags);
+spcg_status_t spcg_solve_wait(spcg_handle_t h, spcg_solve_info_t* info);
+
 /* Single operators of the iterative phase on device vectors (length n), using
  * the same kernels as spcg_solve — for kernel-level parity tests:
  *   spmv:   w = A p          (A the ORIGINAL matrix), *pw = (p,w)

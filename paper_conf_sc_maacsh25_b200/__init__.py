@@ -87,7 +87,7 @@ class SolveInfo(ctypes.Structure):
 EXPORTED = ["spcg_abi_version", "spcg_status_string", "spcg_last_error", "spcg_drop_params_default",
             "spcg_options_default", "spcg_setup", "spcg_get_setup_info", "spcg_solve", "spcg_apply_spmv",
             "spcg_apply_lower", "spcg_apply_upper", "spcg_apply_precond", "spcg_export", "spcg_destroy",
-            "spcg_calibrate"]
+            "spcg_calibrate", "spcg_solve_async", "spcg_solve_wait"]
 
 
 def load(path: str | None = None):
@@ -125,6 +125,10 @@ def load(path: str | None = None):
     lib.spcg_export.restype = I32
     lib.spcg_destroy.argtypes = [V]
     lib.spcg_destroy.restype = None
+    lib.spcg_solve_async.argtypes = [V, P, P, D, I64, ctypes.c_uint32]
+    lib.spcg_solve_async.restype = I32
+    lib.spcg_solve_wait.argtypes = [V, ctypes.POINTER(SolveInfo)]
+    lib.spcg_solve_wait.restype = I32
     lib.spcg_calibrate.argtypes = [I32, ctypes.POINTER(Calib)]
     lib.spcg_calibrate.restype = I32
     if lib.spcg_abi_version() != 1:
@@ -250,6 +254,18 @@ class SPCG:
         st = load().spcg_solve(self._h, b.data_ptr(), x.data_ptr(), float(eps), int(kmax), flags, ctypes.byref(info))
         _check(st, "spcg_solve")
         return x, self._solve_info(info)
+
+    def solve_async(self, b, x, eps=1e-8, kmax=10000):
+        """spcg_solve_async: enqueue on the handle's stream (b, x device tensors kept alive by the caller)."""
+        _check(load().spcg_solve_async(self._h, b.data_ptr(), x.data_ptr(), float(eps), int(kmax), 0),
+               "spcg_solve_async")
+
+    def solve_wait(self):
+        """spcg_solve_wait: finish the in-flight solve, returns its info dict."""
+        info = SolveInfo()
+        st = load().spcg_solve_wait(self._h, ctypes.byref(info))
+        _check(st, "spcg_solve_wait")
+        return self._solve_info(info)
 
     def solve_host(self, b: np.ndarray, eps=1e-8, kmax=10000, x0=None):
         """Host buffers: the library copies b (and x0) in and x out inside the call (e2e path)."""

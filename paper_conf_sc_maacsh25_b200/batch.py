@@ -85,16 +85,75 @@ class Result:
     setup_s: float = 0.0
 
 
-def setup_rank(systems, device: int, mode: str = "alg2", **kw):
-    """Host setup (+ upload when device >= 0) of this rank's systems."""
+def setup_rank(systems, device: int, mode: str = "alg2", lanes: int = 1, sms: int = 148, **kw):
+    """Host setup (+ upload when device >= 0) of this rank's systems.
+
+    lanes > 1: the GPU is split into `lanes` concurrent streams of sms // lanes CTAs
+    each (one persistent CTA per SM, so the cooperative solves in flight always fit
+    the device together); systems go to lanes by LPT on their cost estimate."""
     handles = []
+    lane_of = {}
+    streams = None
+    if lanes > 1 and device >= 0:
+        import torch
+        streams = [torch.cuda.Stream(device) for _ in range(lanes)]
+        for s in systems:
+            if s.cost == 0.0:
+                s.cost = estimate_cost(s)
+        plan, _ = lpt_assign(list(systems), lanes)
+        for li, part in enumerate(plan):
+            for s in part:
+                lane_of[s.index] = li
     for s in systems:
         A = gen.make(s.family, *s.params)
         b, _ = gen.rhs(A)
         t0 = time.perf_counter()
-        h = SPCG(A, mode=mode, K=s.K, device=device, **kw)
+        extra = dict(kw)
+        if streams is not None:
+            extra["stream"] = streams[lane_of[s.index]]
+            extra["parts"] = 1 if A.n <= 16384 else max(1, sms // lanes)
+        h = SPCG(A, mode=mode, K=s.K, device=device, **extra)
+        h.lane = lane_of.get(s.index, 0)
         handles.append((s, A, b, h, time.perf_counter() - t0))
     return handles
+
+
+def solve_rank_concurrent(handles, eps: float = 1e-8, kmax: int = 20000):
+    """All of this rank's systems in flight at once, one stream per lane
+    (spcg_solve_async / spcg_solve_wait).  Returns (results, device makespan ms):
+    events on the default stream fork to every lane and join after the last solve."""
+    import torch
+    dev = handles[0][3].device
+    main = torch.cuda.current_stream(dev)
+    lanes = {}
+    for item in handles:
+        lanes.setdefault(id(item[3].stream), item[3].stream)
+    bufs = []
+    for s, A, b, h, st in handles:       # inputs resident before the timed region
+        with torch.cuda.stream(h.stream):
+            bd = torch.from_numpy(b).to(f"cuda:{dev}", non_blocking=False)
+            bufs.append((bd, torch.empty_like(bd)))
+    torch.cuda.synchronize(dev)
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    t0.record(main)
+    for st_ in lanes.values():
+        st_.wait_event(t0)
+    for (s, A, b, h, st), (bd, xd) in zip(handles, bufs):
+        h.solve_async(bd, xd, eps=eps, kmax=kmax)
+    for st_ in lanes.values():
+        e = torch.cuda.Event()
+        e.record(st_)
+        main.wait_event(e)
+    t1.record(main)
+    out = []
+    for (s, A, b, h, st), (bd, xd) in zip(handles, bufs):
+        info = h.solve_wait()
+        out.append(Result(s.index, s.family, A.n, info["iterations"], info["iter_phase_ms"], info["rnorm"],
+                          info["status"], h.info["chosen_pct"], h.info["levels_L"],
+                          float(xd.double().sum().item()), st))
+    t1.synchronize()
+    return out, float(t0.elapsed_time(t1))
 
 
 def solve_rank(handles, eps: float = 1e-8, kmax: int = 20000, host: bool = False):

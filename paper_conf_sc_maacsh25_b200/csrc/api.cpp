@@ -272,6 +272,33 @@ spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps
     }
 }
 
+spcg_status_t spcg_solve_async(spcg_handle_t h, const double* b, double* x, double eps, int64_t kmax,
+                               uint32_t flags) {
+    if (!h || !b || !x || kmax < 0 || !(eps >= 0.0)) { set_error("bad solve arguments"); return SPCG_ERR_INVALID_ARG; }
+    if (flags & SPCG_HOST_PTRS) { set_error("spcg_solve_async takes device pointers only"); return SPCG_ERR_INVALID_ARG; }
+    if (!h->dev) { set_error("host-only handle"); return SPCG_ERR_NO_DEVICE; }
+    try {
+        return spcg_dev_solve_begin(h->dev, b, x, eps, kmax, (flags & SPCG_USE_X0) != 0);
+    } catch (...) {
+        set_error("unexpected exception in solve");
+        return SPCG_ERR_INTERNAL;
+    }
+}
+
+spcg_status_t spcg_solve_wait(spcg_handle_t h, spcg_solve_info_t* info) {
+    if (!h) return SPCG_ERR_INVALID_ARG;
+    if (!h->dev) { set_error("host-only handle"); return SPCG_ERR_NO_DEVICE; }
+    spcg_solve_info_t tmp{};
+    spcg_solve_info_t* I = info ? info : &tmp;
+    std::memset(I, 0, sizeof *I);
+    try {
+        return spcg_dev_solve_end(h->dev, I, &h->rhist);
+    } catch (...) {
+        set_error("unexpected exception in solve");
+        return SPCG_ERR_INTERNAL;
+    }
+}
+
 spcg_status_t spcg_apply_spmv(spcg_handle_t h, const double* p, double* w, double* pw) {
     if (!h || !p || !w) return SPCG_ERR_INVALID_ARG;
     if (!h->dev) return SPCG_ERR_NO_DEVICE;

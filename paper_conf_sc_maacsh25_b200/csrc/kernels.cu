@@ -1417,6 +1417,12 @@ struct spcg_device_s {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     unsigned long long* trace = nullptr;
     unsigned long long* hb = nullptr;
+    // in-flight solve (spcg_dev_solve_begin .. _end)
+    bool pending = false;
+    double* pend_hist = nullptr;
+    long long pend_cap = 0;
+    double pend_eps = 0.0;
+    void* sc_host = nullptr;       // pinned copy of the device scalars
 };
 
 // debug: copy the heartbeat array while a kernel may still be running (own non-blocking stream)
@@ -1591,6 +1597,8 @@ void spcg_dev_destroy(spcg_device_t* d) {
     if (!d) return;
     cudaSetDevice(d->device);
     cudaStreamSynchronize(d->stream);
+    if (d->pending && d->pend_hist) cudaFree(d->pend_hist);
+    if (d->sc_host) cudaFreeHost(d->sc_host);
     for (void* p : d->allocs) cudaFree(p);
     if (d->ev0) cudaEventDestroy(d->ev0);
     if (d->ev1) cudaEventDestroy(d->ev1);
@@ -1616,9 +1624,13 @@ static spcg_status_t launch(spcg_device_t* d, Params& P) {
     return SPCG_OK;
 }
 
-spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, double eps, int64_t kmax, bool use_x0,
-                             spcg_solve_info_t* info, std::vector<double>* rhist) {
+// Enqueue one solve on the handle's stream and return (asynchronous); the scalar
+// block is copied into pinned host memory on the same stream.
+spcg_status_t spcg_dev_solve_begin(spcg_device_t* d, const double* b, double* x, double eps, int64_t kmax,
+                                   bool use_x0) {
+    if (d->pending) { spcg::set_error("a solve is already in flight on this handle"); return SPCG_ERR_INVALID_ARG; }
     CK(cudaSetDevice(d->device));
+    if (!d->sc_host) CK(cudaMallocHost(&d->sc_host, sizeof(Scal)));
     Params P = d->P;
     P.mode = M_SOLVE;
     P.b = b;
@@ -1638,11 +1650,25 @@ spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, doubl
     spcg_status_t st = launch(d, P);
     if (st != SPCG_OK) { cudaFreeAsync(dh, d->stream); return st; }
     CK(cudaEventRecord(d->ev1, d->stream));
-    Scal sc;
-    CK(cudaMemcpyAsync(&sc, P.sc, sizeof(Scal), cudaMemcpyDeviceToHost, d->stream));
+    CK(cudaMemcpyAsync(d->sc_host, P.sc, sizeof(Scal), cudaMemcpyDeviceToHost, d->stream));
+    d->pending = true;
+    d->pend_hist = dh;
+    d->pend_cap = cap;
+    d->pend_eps = eps;
+    return SPCG_OK;
+}
+
+// Wait for the in-flight solve and fill info (and the residual history).
+spcg_status_t spcg_dev_solve_end(spcg_device_t* d, spcg_solve_info_t* info, std::vector<double>* rhist) {
+    if (!d->pending) { spcg::set_error("no solve in flight on this handle"); return SPCG_ERR_INVALID_ARG; }
+    d->pending = false;
+    CK(cudaSetDevice(d->device));
     CK(cudaStreamSynchronize(d->stream));
+    const Scal sc = *(const Scal*)d->sc_host;
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, d->ev0, d->ev1));
+    const long long cap = d->pend_cap;
+    double* dh = d->pend_hist;
     long long kk = std::min<long long>(sc.k, cap - 1);
     if (rhist) {
         rhist->assign(kk + 1, 0.0);
@@ -1653,7 +1679,7 @@ spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, doubl
     info->iterations = sc.k;
     info->rnorm = std::sqrt(sc.rr);
     info->status = sc.status;
-    info->converged = (sc.status == SPCG_OK && eps > 0.0) ? 1 : 0;
+    info->converged = (sc.status == SPCG_OK && d->pend_eps > 0.0) ? 1 : 0;
     info->iter_phase_ms = ms;
     if (sc.status == SPCG_ERR_INTERNAL) report_abort(d, sc);
     if (d->trace) {
@@ -1667,6 +1693,13 @@ spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, doubl
         }
     }
     return sc.status;
+}
+
+spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, double eps, int64_t kmax, bool use_x0,
+                             spcg_solve_info_t* info, std::vector<double>* rhist) {
+    spcg_status_t st = spcg_dev_solve_begin(d, b, x, eps, kmax, use_x0);
+    if (st != SPCG_OK) return st;
+    return spcg_dev_solve_end(d, info, rhist);
 }
 
 spcg_status_t spcg_dev_apply(spcg_device_t* d, int op, const double* in, double* out, const double* aux,

@@ -159,3 +159,25 @@ def test_calibrate_handoffs_are_ordered():
         assert 0.0 < c[k] < 1e5, (k, c)
     assert c["syncthreads_ns"] < c["flag_same_die_ns"] <= c["flag_cross_die_ns"]
     assert c["flag_same_die_ns"] < c["grid_sync_ns"]
+
+
+def test_async_concurrent_solves_match_sync():
+    """spcg_solve_async / spcg_solve_wait: independent systems in flight on separate
+    streams (C5 lanes) give bitwise the results of spcg_solve."""
+    mats = [gen.make("poisson2d", 40, 33), gen.make("aniso_layered", 96, 64, 4), gen.make("poisson3d", 12, 11, 10)]
+    streams = [torch.cuda.Stream() for _ in mats]
+    hs, bs, xs = [], [], []
+    for A, st in zip(mats, streams):
+        b, _ = gen.rhs(A)
+        hs.append(lib.SPCG(A, mode="alg2", K=0, parts=4, stream=st))
+        bs.append(_dev(b))
+        xs.append(torch.empty_like(bs[-1]))
+    for h, b, x in zip(hs, bs, xs):
+        h.solve_async(b, x, eps=1e-8, kmax=5000)
+    infos = [h.solve_wait() for h in hs]
+    for h, b, x, inf in zip(hs, bs, xs, infos):
+        xr, ir = h.solve(b, eps=1e-8, kmax=5000)
+        assert inf["status"] == 0 and inf["iterations"] == ir["iterations"]
+        assert torch.equal(x, xr)
+    with pytest.raises(lib.SpcgError):
+        hs[0].solve_wait()                       # nothing in flight
