@@ -25,15 +25,16 @@ ap.add_argument("--K", type=int, default=0)
 ap.add_argument("--modes", default="alg2,none")
 ap.add_argument("--sptrsv", default="auto")
 ap.add_argument("--reps", type=int, default=5)
+ap.add_argument("--parts", type=int, default=0)
 ap.add_argument("--tag", default=os.path.basename(os.environ.get("SPCG_LIB", "libspcg.so")))
 a = ap.parse_args()
 
 A = gen.make(a.family, *a.params)
 b, _ = gen.rhs(A)
 bd = torch.from_numpy(b).cuda()
-out = {"tag": a.tag, "family": a.family, "params": a.params, "n": A.n}
+out = {"tag": a.tag, "family": a.family, "params": a.params, "n": A.n, "parts_req": a.parts}
 for mode in a.modes.split(","):
-    h = spcg.SPCG(A, mode=mode, K=a.K, sptrsv=a.sptrsv, device=0)
+    h = spcg.SPCG(A, mode=mode, K=a.K, sptrsv=a.sptrsv, parts=a.parts, device=0)
     x, si = h.solve(bd, eps=1e-8, kmax=10000)
     k_conv = si["iterations"]
     ms = []
