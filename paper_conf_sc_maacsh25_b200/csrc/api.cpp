@@ -250,17 +250,13 @@ spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps
         if (flags & SPCG_HOST_PTRS) {
             // host buffers: H2D of b (and x0), solve, D2H of x — all inside the call
             double* db = nullptr;
-            double* dx = nullptr;
-            st = spcg_dev_copy(h->dev, &db, nullptr, (size_t)h->n * 8, -1);   // alloc
+            st = spcg_dev_copy(h->dev, &db, nullptr, 0, -1);    // the handle's staging buffer (b | x)
             if (st != SPCG_OK) return st;
-            st = spcg_dev_copy(h->dev, &dx, nullptr, (size_t)h->n * 8, -1);
-            if (st != SPCG_OK) { spcg_dev_copy(h->dev, db, nullptr, 0, -2); return st; }
+            double* dx = db + h->n;
             spcg_dev_copy(h->dev, db, b, (size_t)h->n * 8, 1);
             if (flags & SPCG_USE_X0) spcg_dev_copy(h->dev, dx, x, (size_t)h->n * 8, 1);
             st = spcg_dev_solve(h->dev, db, dx, eps, kmax, (flags & SPCG_USE_X0) != 0, I, &h->rhist);
             spcg_dev_copy(h->dev, x, dx, (size_t)h->n * 8, 2);
-            spcg_dev_copy(h->dev, db, nullptr, 0, -2);
-            spcg_dev_copy(h->dev, dx, nullptr, 0, -2);
         } else {
             st = spcg_dev_solve(h->dev, b, x, eps, kmax, (flags & SPCG_USE_X0) != 0, I, &h->rhist);
         }

@@ -1423,6 +1423,9 @@ struct spcg_device_s {
     long long pend_cap = 0;
     double pend_eps = 0.0;
     void* sc_host = nullptr;       // pinned copy of the device scalars
+    double* hist = nullptr;        // residual history buffer (grown on demand, reused)
+    double* stage = nullptr;       // [2n] device copies of host b, x (SPCG_HOST_PTRS), allocated once
+    long long hist_cap = 0;
 };
 
 // debug: copy the heartbeat array while a kernel may still be running (own non-blocking stream)
@@ -1597,7 +1600,8 @@ void spcg_dev_destroy(spcg_device_t* d) {
     if (!d) return;
     cudaSetDevice(d->device);
     cudaStreamSynchronize(d->stream);
-    if (d->pending && d->pend_hist) cudaFree(d->pend_hist);
+    if (d->hist) cudaFree(d->hist);
+    if (d->stage) cudaFree(d->stage);
     if (d->sc_host) cudaFreeHost(d->sc_host);
     for (void* p : d->allocs) cudaFree(p);
     if (d->ev0) cudaEventDestroy(d->ev0);
@@ -1640,15 +1644,19 @@ spcg_status_t spcg_dev_solve_begin(spcg_device_t* d, const double* b, double* x,
     P.use_x0 = use_x0 ? 1 : 0;
     P.epoch = d->epoch;
     d->epoch += (unsigned)(kmax + 3);
-    double* dh = nullptr;
     long long cap = std::min<long long>(kmax + 1, 1 << 20);
-    CK(cudaMallocAsync((void**)&dh, sizeof(double) * cap, d->stream));
+    if (cap > d->hist_cap) {                 // persistent: no allocation on the solve path
+        if (d->hist) { CK(cudaStreamSynchronize(d->stream)); CK(cudaFree(d->hist)); d->hist = nullptr; }
+        d->hist_cap = std::max<long long>(cap, 1024);
+        CK(cudaMalloc((void**)&d->hist, sizeof(double) * d->hist_cap));
+    }
+    double* dh = d->hist;
     P.rhist = dh;
     P.rhist_cap = cap;
     if (d->trace) CK(cudaMemsetAsync(d->trace, 0, sizeof(unsigned long long) * (8 + 4 * (size_t)d->parts + 400), d->stream));
     CK(cudaEventRecord(d->ev0, d->stream));
     spcg_status_t st = launch(d, P);
-    if (st != SPCG_OK) { cudaFreeAsync(dh, d->stream); return st; }
+    if (st != SPCG_OK) return st;
     CK(cudaEventRecord(d->ev1, d->stream));
     CK(cudaMemcpyAsync(d->sc_host, P.sc, sizeof(Scal), cudaMemcpyDeviceToHost, d->stream));
     d->pending = true;
@@ -1674,8 +1682,7 @@ spcg_status_t spcg_dev_solve_end(spcg_device_t* d, spcg_solve_info_t* info, std:
         rhist->assign(kk + 1, 0.0);
         CK(cudaMemcpyAsync(rhist->data(), dh, sizeof(double) * (kk + 1), cudaMemcpyDeviceToHost, d->stream));
     }
-    CK(cudaFreeAsync(dh, d->stream));
-    CK(cudaStreamSynchronize(d->stream));
+    if (rhist) CK(cudaStreamSynchronize(d->stream));
     info->iterations = sc.k;
     info->rnorm = std::sqrt(sc.rr);
     info->status = sc.status;
@@ -1726,13 +1733,9 @@ spcg_status_t spcg_dev_apply(spcg_device_t* d, int op, const double* in, double*
 // kind: 1 H2D, 2 D2H, -1 allocate (dst is void**), -2 free (dst is the pointer)
 spcg_status_t spcg_dev_copy(spcg_device_t* d, void* dst, const void* src, size_t bytes, int kind) {
     CK(cudaSetDevice(d->device));
-    if (kind == -1) {
-        CK(cudaMallocAsync((void**)dst, bytes, d->stream));
-        return SPCG_OK;
-    }
-    if (kind == -2) {
-        CK(cudaFreeAsync(dst, d->stream));
-        CK(cudaStreamSynchronize(d->stream));
+    if (kind == -1) {          // the handle's staging buffer for host b, x: [0, n) and [n, 2n)
+        if (!d->stage) CK(cudaMalloc((void**)&d->stage, 2 * sizeof(double) * (size_t)d->P.n));
+        *(double**)dst = d->stage;
         return SPCG_OK;
     }
     CK(cudaMemcpyAsync(dst, src, bytes, kind == 1 ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToHost, d->stream));
