@@ -540,6 +540,9 @@ constexpr int VEC_WARP0 = POLLER_WARP + NPOLL;
 constexpr int NVEC = 4;
 constexpr int SOLVER_WARP0 = VEC_WARP0 + NVEC;
 static_assert(SOLVER_WARP0 + SPCG_NSOLVER == NWARP, "warp roles must fill the CTA");
+#ifndef SPCG_SOLVER_TREE
+#define SPCG_SOLVER_TREE 0         // 1: fast-path row sum as two interleaved FMA chains (experiment)
+#endif
 #ifndef SPCG_SOLVER_UNROLL
 #define SPCG_SOLVER_UNROLL 4       // record pairs per chunk unrolled in the solver (MAXREC / 2 = all)
 #endif
@@ -818,9 +821,15 @@ __device__ __forceinline__ void prep_record(Prep& X, const ChunkSmem& S, const u
     const int len = meta_len(X.meta), ne = meta_ne(X.meta);
     const uint8_t* sp = X.p + SPCG_REC_HDR + 4 * lane;
     const uint8_t* vp = X.p + SPCG_REC_HDR + 128 * X.wd + 8 * lane;
+    // ring entries in registers.  Only the warp-uniform width guards the loads: the
+    // layout stores padding entries (k >= len, padding lanes) as (slot 0, 0.0), so
+    // they add nothing; cross-CTA entries (k < ne, negative slots) exist only in
+    // REC_EXT records, whose path masks them (solve_record).
+    (void)len;
+    (void)ne;
 #pragma unroll
     for (int k = 0; k < WP; ++k) {
-        const bool on = k >= ne && k < len && k < X.wd;     // ring entries in registers
+        const bool on = k < X.wd;
         X.sidx[k] = on ? *(const int*)(sp + 128 * k) : 0;
         X.v[k] = on ? *(const double*)(vp + 256 * k) : 0.0;
     }
@@ -901,9 +910,22 @@ __device__ __forceinline__ void solve_record(const SolveCtx& C, const Prep& X, i
         double d[WP];
 #pragma unroll
         for (int k = 0; k < WP; ++k) d[k] = C.yring[X.sidx[k]];
-        double acc = X.vec;
+        double acc;
+        if (SPCG_SOLVER_TREE) {
+            // two independent FMA chains then one add: depth 3 instead of WP = 4 on the
+            // record-to-record dependency path (rounding order differs from the chain)
+            double a0 = fma(-X.v[0], d[0], X.vec), a1 = -X.v[1] * d[1];
 #pragma unroll
-        for (int k = 0; k < WP; ++k) acc = fma(-X.v[k], d[k], acc);   // v = 0 off-entry
+            for (int k = 2; k < WP; ++k) {
+                if (k & 1) a1 = fma(-X.v[k], d[k], a1);
+                else a0 = fma(-X.v[k], d[k], a0);
+            }
+            acc = a0 + a1;
+        } else {
+            acc = X.vec;
+#pragma unroll
+            for (int k = 0; k < WP; ++k) acc = fma(-X.v[k], d[k], acc);   // v = 0 off-entry
+        }
         finish_row<UPPER, PRO>(C, X.row, X.meta, acc, X.dinv, X.aux, rz);
         acc_carry = acc;
     } else if ((X.fl & (REC_FIRST | REC_WIDE)) == REC_FIRST) {
@@ -918,10 +940,10 @@ __device__ __forceinline__ void solve_record(const SolveCtx& C, const Prep& X, i
             if (ne > 0) e = lds_volatile(side_ext(*C.S, slot, X.r) + lane);
             double d[WP];
 #pragma unroll
-            for (int k = 0; k < WP; ++k) d[k] = C.yring[X.sidx[k]];
+            for (int k = 0; k < WP; ++k) d[k] = C.yring[k < ne ? 0 : X.sidx[k]];
             double acc = X.vec - e;
 #pragma unroll
-            for (int k = 0; k < WP; ++k) acc = fma(-X.v[k], d[k], acc);
+            for (int k = 0; k < WP; ++k) acc = fma(k < ne ? 0.0 : -X.v[k], d[k], acc);
             finish_row<UPPER, PRO>(C, X.row, X.meta, acc, X.dinv, X.aux, rz);
             acc_carry = acc;
         } else {
@@ -962,6 +984,8 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
         if (dbg) t_wait += clock64() - tw;
         const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
         const int nrec = *(const uint16_t*)ch;
+        // progress for the pollers, once per chunk (the first record the solver is on)
+        if (lane == 0) S.progress[0] = recn;
         Prep A, B;
         if (nrec > 0) prep_record<UPPER>(A, S, ch, slot, 0, lane);
 #pragma unroll kSolverUnroll
@@ -970,14 +994,12 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
             if (r + 1 < nrec) prep_record<UPPER>(B, S, ch, slot, r + 1, lane);
             if (dbg) { t_prep += clock64() - tp; tp = clock64(); }
             if (r < nrec) {
-                if (lane == 0) S.progress[0] = recn + r;
                 solve_record<UPPER, PRO>(C, A, slot, lane, acc_carry, rz);
             }
             if (dbg) { t_solve += clock64() - tp; tp = clock64(); }
             if (r + 2 < nrec) prep_record<UPPER>(A, S, ch, slot, r + 2, lane);
             if (dbg) { t_prep += clock64() - tp; tp = clock64(); }
             if (r + 1 < nrec) {
-                if (lane == 0) S.progress[0] = recn + r + 1;
                 solve_record<UPPER, PRO>(C, B, slot, lane, acc_carry, rz);
             }
             if (dbg) t_solve += clock64() - tp;

@@ -1,0 +1,5 @@
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 600 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -2 gpurun_out/pytest_gpu.log
+timeout 300 python tools/exp_iter.py aniso_layered 2048 2048 4 --k 30 --modes alg2 >> gpurun_out/exp9.jsonl 2>>gpurun_out/exp9.err
+timeout 300 python tools/exp_iter.py poisson3d 64 64 64 --k 30 --modes alg2 >> gpurun_out/exp9.jsonl 2>>gpurun_out/exp9.err
+timeout 300 python tools/diag.py aniso_layered 2048 2048 4 --k 10 >> gpurun_out/diag.jsonl 2>>gpurun_out/diag.err
