@@ -374,9 +374,13 @@ def run_batch(args, ws, rank, local):
     sms = torch.cuda.get_device_properties(local).multi_processor_count
     hs = batch.setup_rank(plan[rank], device=local, lanes=args.lanes, sms=sms)
 
+    order = {}
+
     def step():
         if args.lanes > 1:
-            return batch.solve_rank_concurrent(hs)
+            r, mk = batch.solve_rank_dynamic(hs, args.lanes, order=order or None)
+            order.update({x.index: x.iter_phase_ms for x in r})      # longest first next time
+            return r, mk
         r = batch.solve_rank(hs)
         return r, sum(x.iter_phase_ms for x in r)
 
@@ -422,8 +426,9 @@ def run_batch(args, ws, rank, local):
                 "ms_per_step": ms, "higher_is_better": False, "scaling": "strong", "vs_baseline": None,
                 "dtype": "f64", "data": "synthetic",
                 "config": {"workload": WORKLOADS["C5"], "systems": len(systems), "eps": EPS, "lanes": args.lanes,
-                           "makespan": ("device events fork/join around all of the rank's solves in flight on "
-                                        f"{args.lanes} streams x {sms // args.lanes} CTAs" if args.lanes > 1 else
+                           "makespan": ("device events fork/join around the rank's solves, list-scheduled longest "
+                                        f"first (previous step's times) onto {args.lanes} streams x "
+                                        f"{sms // args.lanes} CTAs" if args.lanes > 1 else
                                         "sum of the rank's device-timed solves (back to back)") +
                                        "; max over ranks",
                            "l2": "no flush: 64 different systems run back to back (working set >> L2)"},

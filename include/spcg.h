@@ -195,6 +195,10 @@ spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps
 spcg_status_t spcg_solve_async(spcg_handle_t h, const double* b, double* x, double eps, int64_t kmax,
                                uint32_t flags);
 spcg_status_t spcg_solve_wait(spcg_handle_t h, spcg_solve_info_t* info);
+/* Moves the handle's work to another cudaStream_t (a batch scheduler hands
+ * systems to whichever lane is free).  Synchronises the old stream first;
+ * INVALID_ARG while a solve is in flight. */
+spcg_status_t spcg_set_stream(spcg_handle_t h, void* stream);
 
 /* Single operators of the iterative phase on device vectors (length n), using
  * the same kernels as spcg_solve — for kernel-level parity tests:

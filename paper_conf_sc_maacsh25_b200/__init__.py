@@ -87,7 +87,7 @@ class SolveInfo(ctypes.Structure):
 EXPORTED = ["spcg_abi_version", "spcg_status_string", "spcg_last_error", "spcg_drop_params_default",
             "spcg_options_default", "spcg_setup", "spcg_get_setup_info", "spcg_solve", "spcg_apply_spmv",
             "spcg_apply_lower", "spcg_apply_upper", "spcg_apply_precond", "spcg_export", "spcg_destroy",
-            "spcg_calibrate", "spcg_solve_async", "spcg_solve_wait"]
+            "spcg_calibrate", "spcg_solve_async", "spcg_solve_wait", "spcg_set_stream"]
 
 
 def load(path: str | None = None):
@@ -129,6 +129,8 @@ def load(path: str | None = None):
     lib.spcg_solve_async.restype = I32
     lib.spcg_solve_wait.argtypes = [V, ctypes.POINTER(SolveInfo)]
     lib.spcg_solve_wait.restype = I32
+    lib.spcg_set_stream.argtypes = [V, V]
+    lib.spcg_set_stream.restype = I32
     lib.spcg_calibrate.argtypes = [I32, ctypes.POINTER(Calib)]
     lib.spcg_calibrate.restype = I32
     if lib.spcg_abi_version() != 1:
@@ -259,6 +261,11 @@ class SPCG:
         """spcg_solve_async: enqueue on the handle's stream (b, x device tensors kept alive by the caller)."""
         _check(load().spcg_solve_async(self._h, b.data_ptr(), x.data_ptr(), float(eps), int(kmax), 0),
                "spcg_solve_async")
+
+    def set_stream(self, stream):
+        """spcg_set_stream: later solves of this handle run on `stream` (a torch.cuda.Stream)."""
+        _check(load().spcg_set_stream(self._h, stream.cuda_stream), "spcg_set_stream")
+        self.stream = stream
 
     def solve_wait(self):
         """spcg_solve_wait: finish the in-flight solve, returns its info dict."""

@@ -118,6 +118,67 @@ def setup_rank(systems, device: int, mode: str = "alg2", lanes: int = 1, sms: in
     return handles
 
 
+def solve_rank_dynamic(handles, lanes: int, eps: float = 1e-8, kmax: int = 20000, order=None):
+    """List scheduling over `lanes` concurrent streams: the systems, longest first
+    (`order`: expected solve ms per system index, e.g. the previous step's), go to
+    whichever lane frees up first (spcg_set_stream + spcg_solve_async; lane
+    completion seen through an event query).  Every handle was set up with
+    sms // lanes CTAs, so the cooperative solves in flight always fit the GPU
+    together.  Returns (results, device makespan ms from fork/join events)."""
+    import torch
+    dev = handles[0][3].device
+    main = torch.cuda.current_stream(dev)
+    streams = [torch.cuda.Stream(dev) for _ in range(lanes)]
+    bufs = {}
+    for s, A, b, h, st in handles:       # inputs resident before the timed region
+        bd = torch.from_numpy(b).to(f"cuda:{dev}")
+        bufs[s.index] = (bd, torch.empty_like(bd))
+    torch.cuda.synchronize(dev)
+    for s, A, b, h, st in handles:
+        h.set_stream(streams[0])
+    key = (lambda it: -order[it[0].index]) if order else (lambda it: -(it[0].cost or estimate_cost(it[0])))
+    queue = sorted(handles, key=key)
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    t0.record(main)
+    for st_ in streams:
+        st_.wait_event(t0)
+    running = {}
+    out = []
+
+    def launch(item, lane):
+        s, A, b, h, st = item
+        h.set_stream(streams[lane])
+        bd, xd = bufs[s.index]
+        h.solve_async(bd, xd, eps=eps, kmax=kmax)
+        ev = torch.cuda.Event()
+        ev.record(streams[lane])
+        running[lane] = (item, ev)
+
+    for lane in range(min(lanes, len(queue))):
+        launch(queue.pop(0), lane)
+    while running:
+        done = [lane for lane, (_, ev) in running.items() if ev.query()]
+        if not done:
+            time.sleep(2e-5)
+            continue
+        for lane in done:
+            (s, A, b, h, st), _ = running.pop(lane)
+            info = h.solve_wait()
+            out.append(Result(s.index, s.family, A.n, info["iterations"], info["iter_phase_ms"], info["rnorm"],
+                              info["status"], h.info["chosen_pct"], h.info["levels_L"],
+                              float(bufs[s.index][1].double().sum().item()), st))
+            if queue:
+                launch(queue.pop(0), lane)
+    for st_ in streams:
+        e = torch.cuda.Event()
+        e.record(st_)
+        main.wait_event(e)
+    t1.record(main)
+    t1.synchronize()
+    return sorted(out, key=lambda r: r.index), float(t0.elapsed_time(t1))
+
+
 def solve_rank_concurrent(handles, eps: float = 1e-8, kmax: int = 20000):
     """All of this rank's systems in flight at once, one stream per lane
     (spcg_solve_async / spcg_solve_wait).  Returns (results, device makespan ms):

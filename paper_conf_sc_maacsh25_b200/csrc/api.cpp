@@ -281,6 +281,12 @@ spcg_status_t spcg_solve_async(spcg_handle_t h, const double* b, double* x, doub
     }
 }
 
+spcg_status_t spcg_set_stream(spcg_handle_t h, void* stream) {
+    if (!h) return SPCG_ERR_INVALID_ARG;
+    if (!h->dev) { set_error("host-only handle"); return SPCG_ERR_NO_DEVICE; }
+    return spcg_dev_set_stream(h->dev, stream);
+}
+
 spcg_status_t spcg_solve_wait(spcg_handle_t h, spcg_solve_info_t* info) {
     if (!h) return SPCG_ERR_INVALID_ARG;
     if (!h->dev) { set_error("host-only handle"); return SPCG_ERR_NO_DEVICE; }

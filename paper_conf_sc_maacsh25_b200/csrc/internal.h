@@ -138,6 +138,7 @@ spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, doubl
                              bool use_x0, spcg_solve_info_t* info, std::vector<double>* rhist);
 spcg_status_t spcg_dev_solve_begin(spcg_device_t* d, const double* b, double* x, double eps, int64_t kmax,
                                    bool use_x0);
+spcg_status_t spcg_dev_set_stream(spcg_device_t* d, void* stream);
 spcg_status_t spcg_dev_solve_end(spcg_device_t* d, spcg_solve_info_t* info, std::vector<double>* rhist);
 spcg_status_t spcg_dev_apply(spcg_device_t* d, int op, const double* in, double* out,
                              const double* aux, double* scalar_out);

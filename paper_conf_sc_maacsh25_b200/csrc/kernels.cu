@@ -1688,6 +1688,16 @@ spcg_status_t spcg_dev_solve_begin(spcg_device_t* d, const double* b, double* x,
     return SPCG_OK;
 }
 
+// Rebind the handle to another stream (work already queued on the old one is
+// finished first, so the new stream never overtakes it).
+spcg_status_t spcg_dev_set_stream(spcg_device_t* d, void* stream) {
+    if (d->pending) { spcg::set_error("cannot rebind the stream of a handle with a solve in flight"); return SPCG_ERR_INVALID_ARG; }
+    CK(cudaSetDevice(d->device));
+    CK(cudaStreamSynchronize(d->stream));
+    d->stream = (cudaStream_t)stream;
+    return SPCG_OK;
+}
+
 // Wait for the in-flight solve and fill info (and the residual history).
 spcg_status_t spcg_dev_solve_end(spcg_device_t* d, spcg_solve_info_t* info, std::vector<double>* rhist) {
     if (!d->pending) { spcg::set_error("no solve in flight on this handle"); return SPCG_ERR_INVALID_ARG; }
