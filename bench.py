@@ -59,15 +59,20 @@ def _peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def _ncu_traffic(workload: str, impl: str):
-    """dram bytes per launch of the persistent kernel from the committed ncu summary."""
+def _ncu_traffic(workload: str, impl: str, iterations: int):
+    """DRAM bytes (read + write) of the persistent kernel per launch of THIS bench's solve:
+    the committed ncu capture's bytes per iteration (launch bytes / (k_capture + 1 for the
+    prologue)) x (iterations + 1)."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if not os.path.exists(p):
         return None
     try:
         d = json.load(open(p))
         e = d.get(workload, {}).get(impl)
-        return None if e is None else float(e["dram_bytes_per_launch"])
+        if e is None:
+            return None
+        per = float(e.get("dram_bytes_per_iter", e["dram_bytes_per_launch"]))
+        return per * (iterations + 1) if "dram_bytes_per_iter" in e else per
     except Exception:
         return None
 
@@ -295,7 +300,7 @@ def main():
     s_bi, p_bi = si["algo_bytes_per_iter"], pi["algo_bytes_per_iter"]
     s_gbs = s_bi * s["k"] / (s_ms * 1e-3) / 1e9
     p_gbs = p_bi * p["k"] / (p_ms * 1e-3) / 1e9
-    traffic = _ncu_traffic(name, "spcg")
+    traffic = _ncu_traffic(name, "spcg", s["k"])
     cpu = None
     if not args.no_cpu_baseline:
         o = run_oracle(name, A, b, 2, 0, budget_s=20.0, k_hint={"alg2": s["k"], "none": p["k"]})
