@@ -159,12 +159,13 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             strategy = (h->identity || wl <= (double)SPCG_WCAP) ? SPCG_SPTRSV_CHUNKED : SPCG_SPTRSV_LEVEL;
         }
         if (strategy < 1 || strategy > 3) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }
+        const int slots = sms * spcg_dev_ctas_per_sm();        // co-resident persistent CTAs
         int parts = opt.parts;
-        if (parts <= 0) parts = h->n <= 16384 ? 1 : sms;
-        parts = std::max(1, std::min<int>(parts, sms));
+        if (parts <= 0) parts = h->n <= 16384 ? 1 : slots;
+        parts = std::max(1, std::min<int>(parts, slots));
         if ((int64_t)parts > h->n) parts = (int)h->n;
         build_spmv_layout(h->A, h->lay.A);
-        build_tri_layouts(h->F, strategy, parts, 16384, h->lay);
+        build_tri_layouts(h->F, strategy, parts, spcg_dev_ring_max(), h->lay);
         double t5 = now_ms();
         int64_t bytes = 0;
         if (opt.device >= 0) {

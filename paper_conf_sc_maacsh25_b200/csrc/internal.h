@@ -93,7 +93,10 @@ struct SpmvLayout {                // SELL-32 of the original A, natural row ord
 // slice records, L section then U section, cut into CHUNK-byte chunks that the
 // kernel copies into a shared-memory ring with cp.async.bulk.
 constexpr int SPCG_CHUNK_BYTES = 4096;
-constexpr int SPCG_NCHUNK = 8;          // ring slots
+#ifndef SPCG_NCHUNK_SLOTS
+#define SPCG_NCHUNK_SLOTS 8
+#endif
+constexpr int SPCG_NCHUNK = SPCG_NCHUNK_SLOTS;   // chunk ring slots in shared memory (kernel side)
 constexpr int SPCG_MAXREC = 8;          // records per chunk (side-data slots)
 constexpr int SPCG_WCAP = 8;            // entry columns per record
 constexpr int SPCG_NSOLVER = 1;         // solver warps per CTA (one software-pipelined chain)
@@ -138,6 +141,8 @@ spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, doubl
                              bool use_x0, spcg_solve_info_t* info, std::vector<double>* rhist);
 spcg_status_t spcg_dev_solve_begin(spcg_device_t* d, const double* b, double* x, double eps, int64_t kmax,
                                    bool use_x0);
+int spcg_dev_ctas_per_sm();
+int spcg_dev_ring_max();
 spcg_status_t spcg_dev_set_stream(spcg_device_t* d, void* stream);
 spcg_status_t spcg_dev_solve_end(spcg_device_t* d, spcg_solve_info_t* info, std::vector<double>* rhist);
 spcg_status_t spcg_dev_apply(spcg_device_t* d, int op, const double* in, double* out,

@@ -37,9 +37,15 @@ using namespace spcg;
 
 namespace {
 
-constexpr int BLOCK = 256;
+#ifndef SPCG_BLOCK
+#define SPCG_BLOCK 256            // threads per persistent CTA (128: 4-warp CTAs, two per SM)
+#endif
+constexpr int BLOCK = SPCG_BLOCK;
 #ifndef SPCG_CTAS_PER_SM
-#define SPCG_CTAS_PER_SM 1        // persistent CTAs per SM (2: two independent chains per SM, <= 128 registers)
+#define SPCG_CTAS_PER_SM (SPCG_BLOCK == 128 ? 2 : 1)   // persistent CTAs per SM (independent chains per SM)
+#endif
+#ifndef SPCG_RING_MAX
+#define SPCG_RING_MAX (SPCG_CTAS_PER_SM > 1 ? 4096 : 16384)   // shared-memory ring entries (power of two)
 #endif
 constexpr int NWARP = BLOCK / 32;
 constexpr long long SPIN_TIMEOUT_CYC = 8ll * 1000 * 1000 * 1000;            // ~4 s of SM cycles: abort, never hang
@@ -535,9 +541,9 @@ __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const doub
 //                 ahead so only ring gather -> FMA -> store sits on the critical path
 constexpr int PRODUCER_WARP = 0;
 constexpr int POLLER_WARP = 1;
-constexpr int NPOLL = 2;                          // poller warps (records alternate)
+constexpr int NPOLL = NWARP >= 8 ? 2 : 1;         // poller warps (records alternate)
 constexpr int VEC_WARP0 = POLLER_WARP + NPOLL;
-constexpr int NVEC = 4;
+constexpr int NVEC = NWARP - 2 - NPOLL;           // 4 (8 warps) or 1 (4 warps)
 constexpr int SOLVER_WARP0 = VEC_WARP0 + NVEC;
 static_assert(SOLVER_WARP0 + SPCG_NSOLVER == NWARP, "warp roles must fill the CTA");
 #ifndef SPCG_SOLVER_TREE
@@ -1509,6 +1515,10 @@ static spcg_status_t upload_tri(spcg_device_t* d, const spcg::TriLayout& T, DevT
     return SPCG_OK;
 }
 
+// launch geometry the host setup must use (compile-time knobs of this build)
+int spcg_dev_ctas_per_sm() { return SPCG_CTAS_PER_SM; }
+int spcg_dev_ring_max() { return SPCG_RING_MAX; }
+
 extern "C" int spcg_dev_sm_count(int device) {
     cudaDeviceProp prop;
     if (cudaSetDevice(device) != cudaSuccess) { spcg::set_error("cudaSetDevice failed"); return -1; }
@@ -1576,8 +1586,8 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
     }
     d->smem = lay.strategy == ST_CHUNKED ? chunked_smem_bytes(lay.ring) : 0;
     void* kfn = pick_kernel(d->strategy);
-    // one attribute value for every handle: the largest ring any layout builds (16384 entries)
-    const int smem_max = lay.strategy == ST_CHUNKED ? (int)chunked_smem_bytes(16384) : 0;
+    // one attribute value for every handle: the largest ring any layout builds
+    const int smem_max = lay.strategy == ST_CHUNKED ? (int)chunked_smem_bytes(SPCG_RING_MAX) : 0;
     if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max) != cudaSuccess) {
         spcg::set_error("cannot reserve shared memory for the ring");
         spcg_dev_destroy(d);
