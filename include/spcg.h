@@ -196,8 +196,9 @@ spcg_status_t spcg_solve_async(spcg_handle_t h, const double* b, double* x, doub
                                uint32_t flags);
 spcg_status_t spcg_solve_wait(spcg_handle_t h, spcg_solve_info_t* info);
 /* Moves the handle's work to another cudaStream_t (a batch scheduler hands
- * systems to whichever lane is free).  Synchronises the old stream first;
- * INVALID_ARG while a solve is in flight. */
+ * systems to whichever lane is free).  The new stream waits on the device for
+ * the work already queued on the old one (no host blocking); INVALID_ARG while
+ * a solve is in flight. */
 spcg_status_t spcg_set_stream(spcg_handle_t h, void* stream);
 
 /* Single operators of the iterative phase on device vectors (length n), using

@@ -1443,6 +1443,7 @@ struct spcg_device_s {
     int64_t bytes = 0;
     unsigned epoch = 1;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    cudaEvent_t ev_bind = nullptr;   // spcg_dev_set_stream ordering
     unsigned long long* trace = nullptr;
     unsigned long long* hb = nullptr;
     // in-flight solve (spcg_dev_solve_begin .. _end)
@@ -1637,6 +1638,7 @@ void spcg_dev_destroy(spcg_device_t* d) {
     if (d->sc_host) cudaFreeHost(d->sc_host);
     for (void* p : d->allocs) cudaFree(p);
     if (d->ev0) cudaEventDestroy(d->ev0);
+    if (d->ev_bind) cudaEventDestroy(d->ev_bind);
     if (d->ev1) cudaEventDestroy(d->ev1);
     delete d;
 }
@@ -1698,12 +1700,16 @@ spcg_status_t spcg_dev_solve_begin(spcg_device_t* d, const double* b, double* x,
     return SPCG_OK;
 }
 
-// Rebind the handle to another stream (work already queued on the old one is
-// finished first, so the new stream never overtakes it).
+// Rebind the handle to another stream.  The new stream waits (on the device,
+// through an event) for the work already queued on the old one, so it never
+// overtakes it; the host does not block.
 spcg_status_t spcg_dev_set_stream(spcg_device_t* d, void* stream) {
     if (d->pending) { spcg::set_error("cannot rebind the stream of a handle with a solve in flight"); return SPCG_ERR_INVALID_ARG; }
+    if ((cudaStream_t)stream == d->stream) return SPCG_OK;
     CK(cudaSetDevice(d->device));
-    CK(cudaStreamSynchronize(d->stream));
+    if (!d->ev_bind) CK(cudaEventCreateWithFlags(&d->ev_bind, cudaEventDisableTiming));
+    CK(cudaEventRecord(d->ev_bind, d->stream));
+    CK(cudaStreamWaitEvent((cudaStream_t)stream, d->ev_bind, 0));
     d->stream = (cudaStream_t)stream;
     return SPCG_OK;
 }
