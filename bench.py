@@ -180,6 +180,8 @@ def main():
     ap.add_argument("--batch-count", type=int, default=64)
     ap.add_argument("--lanes", type=int, default=4,
                     help="C5: concurrent streams per GPU (each with SMs/lanes persistent CTAs)")
+    ap.add_argument("--sched", default="static", choices=["static", "dynamic"],
+                    help="C5 lanes: static LPT lanes, all enqueued up front (default), or host list scheduling")
     ap.add_argument("--sweep", default=None,
                     help="comma list of fixed drop ratios t%% timed beside Alg. 2 and PCG (default: 1,5,10 for C4)")
     args = ap.parse_args()
@@ -382,10 +384,12 @@ def run_batch(args, ws, rank, local):
     order = {}
 
     def step():
-        if args.lanes > 1:
+        if args.lanes > 1 and args.sched == "dynamic":
             r, mk = batch.solve_rank_dynamic(hs, args.lanes, order=order or None)
             order.update({x.index: x.iter_phase_ms for x in r})      # longest first next time
             return r, mk
+        if args.lanes > 1:
+            return batch.solve_rank_concurrent(hs)
         r = batch.solve_rank(hs)
         return r, sum(x.iter_phase_ms for x in r)
 
@@ -431,9 +435,8 @@ def run_batch(args, ws, rank, local):
                 "ms_per_step": ms, "higher_is_better": False, "scaling": "strong", "vs_baseline": None,
                 "dtype": "f64", "data": "synthetic",
                 "config": {"workload": WORKLOADS["C5"], "systems": len(systems), "eps": EPS, "lanes": args.lanes,
-                           "makespan": ("device events fork/join around the rank's solves, list-scheduled longest "
-                                        f"first (previous step's times) onto {args.lanes} streams x "
-                                        f"{sms // args.lanes} CTAs" if args.lanes > 1 else
+                           "makespan": (f"device events fork/join around the rank's solves ({args.sched} lanes: "
+                                        f"{args.lanes} streams x {sms // args.lanes} CTAs)" if args.lanes > 1 else
                                         "sum of the rank's device-timed solves (back to back)") +
                                        "; max over ranks",
                            "l2": "no flush: 64 different systems run back to back (working set >> L2)"},

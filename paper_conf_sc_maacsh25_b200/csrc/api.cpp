@@ -150,13 +150,14 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         }
         // AUTO: the chunked executor streams thread-per-row records of <= SPCG_WCAP entry
         // columns; rows wider than that (ILU(K) fill of 3-D stencils: ~57 entries per L row
-        // for 27-point ILU(2)) need continuation records on the serial chain, where the
-        // level-scheduled executor (grid barrier per wavefront, the design of [36]) is faster
-        // (measured: FEM 48^3 ILU(2) 26 vs 31.5 ms per iteration).
+        // for 27-point ILU(2)) need continuation records on the serial chain.  For those the
+        // sync-free executor with one warp per row is fastest (measured, FEM 48^3 ILU(2), per
+        // iteration: chunked 31.5 ms, level warp-per-row 6.3 ms, sync-free warp-per-row
+        // 2.2 ms).
         int strategy = opt.sptrsv;
         if (strategy == SPCG_SPTRSV_AUTO) {
             const double wl = h->n > 0 ? (double)h->F.L.nnz() / (double)h->n : 0.0;
-            strategy = (h->identity || wl <= (double)SPCG_WCAP) ? SPCG_SPTRSV_CHUNKED : SPCG_SPTRSV_LEVEL;
+            strategy = (h->identity || wl <= (double)SPCG_WCAP) ? SPCG_SPTRSV_CHUNKED : SPCG_SPTRSV_SYNCFREE;
         }
         if (strategy < 1 || strategy > 3) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }
         const int slots = sms * spcg_dev_ctas_per_sm();        // co-resident persistent CTAs

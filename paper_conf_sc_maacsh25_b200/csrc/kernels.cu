@@ -506,6 +506,72 @@ __device__ void tri_level_wide(const Params& P, const DevTri& T, int kind, const
     }
 }
 
+// SYNCFREE executor, wide rows: the warp-per-row CSR of tri_level_wide, but no
+// barriers — rows in execution (level) order are dealt round-robin to all warps
+// of the grid; each lane waits on the LL ready flags of its dependencies, the
+// warp reduces, lane 0 publishes the row's value with its flag.  Deadlock-free
+// because every dependency has a lower position and all warps are co-resident.
+template <bool UPPER>
+__device__ void tri_syncfree_wide(const Params& P, const DevTri& T, int kind, const double* in, double* out,
+                                  const double* rdot, uint4* mb, unsigned ep, double alpha, double& acc_dot) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t W = (int64_t)gridDim.x * NWARP;
+    for (int64_t q = (int64_t)blockIdx.x * NWARP + warp; q < P.n; q += W) {
+        const int row = __ldg(T.wrow + q);
+        const int64_t e0 = __ldg(T.wptr + q), e1 = __ldg(T.wptr + q + 1);
+        double r0 = 0.0, w0 = 0.0, x0 = 0.0, p0v = 0.0, a0 = 0.0, dv = 1.0;
+        if (lane == 0) {
+            if (!UPPER) {
+                if (kind == K_ITER) { r0 = __ldcg(P.r + row); w0 = __ldcg(P.w + row); x0 = __ldcg(P.x + row); p0v = __ldcg(P.p + row); }
+                else r0 = __ldcg(in + row);
+            } else {
+                r0 = __ldcg(in + row);
+                if (rdot) a0 = __ldcg(rdot + row);
+                dv = __ldg(T.wdinv + q);
+            }
+        }
+        // all of this lane's (index, value) pairs first, then the flag waits
+        int c[WPF];
+        double v[WPF];
+#pragma unroll
+        for (int u = 0; u < WPF; ++u) {
+            const int64_t e = e0 + lane + 32 * u;
+            c[u] = e < e1 ? __ldg(T.wcol + e) : -1;
+            v[u] = e < e1 ? __ldg(T.wval + e) : 0.0;
+        }
+        double part = 0.0;
+#pragma unroll
+        for (int u = 0; u < WPF; ++u)
+            if (c[u] >= 0) part = fma(v[u], ll_wait(mb + c[u], ep, P.sc), part);
+        for (int64_t e = e0 + lane + 32 * WPF; e < e1; e += 32)
+            part = fma(__ldg(T.wval + e), ll_wait(mb + __ldg(T.wcol + e), ep, P.sc), part);
+        part = warp_sum(part);
+        if (lane == 0) {
+            double acc;
+            if (!UPPER) {
+                double ri = r0;
+                if (kind == K_ITER) {
+                    ri = r0 - alpha * w0;
+                    P.r[row] = ri;
+                    P.x[row] = x0 + alpha * p0v;
+                } else if (kind == K_PRO) {
+                    if (in != P.r) P.r[row] = ri;
+                    if (!P.use_x0) P.x[row] = 0.0;
+                }
+                acc_dot = fma(ri, ri, acc_dot);
+                acc = ri - part;
+            } else {
+                acc = (r0 - part) * dv;
+                if (rdot) acc_dot = fma(a0, acc, acc_dot);
+                if (kind == K_PRO) P.p[row] = acc;
+            }
+            out[row] = acc;
+            ll_store(mb + row, acc, ep);
+        }
+        __syncwarp();
+    }
+}
+
 template <int STRAT, bool UPPER>
 __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const double* in, double* out,
                           const double* rdot, uint4* mb, unsigned ep, double alpha, double& acc_dot,
@@ -513,6 +579,8 @@ __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const doub
     const int warp = threadIdx.x >> 5;
     if (STRAT == ST_LEVEL && T.wide) {
         tri_level_wide<UPPER>(P, T, kind, in, out, rdot, alpha, acc_dot, gen);
+    } else if (STRAT == ST_SYNCFREE && T.wide) {
+        tri_syncfree_wide<UPPER>(P, T, kind, in, out, rdot, mb, ep, alpha, acc_dot);
     } else if (STRAT == ST_LEVEL) {
         const int64_t W = (int64_t)gridDim.x * NWARP;
         const int64_t gw = (int64_t)blockIdx.x * NWARP + warp;

@@ -103,7 +103,8 @@ static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev,
     {
         int64_t deps = 0;
         for (int64_t i = 0; i < n; ++i) deps += dep_end(i) - dep_begin(i);
-        T.wide = strategy == SPCG_SPTRSV_LEVEL && n > 0 && (double)deps / (double)n > (double)SPCG_WCAP;
+        T.wide = (strategy == SPCG_SPTRSV_LEVEL || strategy == SPCG_SPTRSV_SYNCFREE) && n > 0 &&
+                 (double)deps / (double)n > (double)SPCG_WCAP;
         if (T.wide) {
             T.wrow.assign(order.begin(), order.end());
             T.wgptr.assign(grp_rows_ptr.begin(), grp_rows_ptr.end());
