@@ -322,6 +322,8 @@ def main():
         "iterations": s["k"], "ms_per_iter": s_ms / max(s["k"], 1),
         "hbm_gbs_per_iter": s_gbs, "algo_bytes_per_iter": s_bi,
         "levels": {"L": si["levels_L"], "U": si["levels_U"], "w_A": si["w_A"], "w_Ahat": si["w_Ahat"]},
+        "nnz": {"A": si["nnz_A"], "Ahat": si["nnz_Ahat"], "L_s": si["nnz_L"], "U": si["nnz_U"]},
+        "ncu_dram_gbs": None if traffic is None else traffic / (s_ms * 1e-3) / 1e9,
         "pcg": {"value": p_ms, "iterations": p["k"], "ms_per_iter": p_ms / max(p["k"], 1), "hbm_gbs_per_iter": p_gbs,
                 "algo_bytes_per_iter": p_bi, "levels": {"L": pi["levels_L"], "U": pi["levels_U"]}},
         "sweep": sweep or None,

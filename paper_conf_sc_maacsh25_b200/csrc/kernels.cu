@@ -724,6 +724,7 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned by
 }
 
 __device__ ChunkSmem chunk_smem(double* dyn, int ring) {
+    // the host guarantees ring >= 16 and a power of two (layout.cpp): chunks stay 128-byte aligned
     ChunkSmem S;
     uint8_t* base = (uint8_t*)dyn;
     S.yring = dyn;

@@ -103,8 +103,11 @@ static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev,
     {
         int64_t deps = 0;
         for (int64_t i = 0; i < n; ++i) deps += dep_end(i) - dep_begin(i);
+        // experiment knob: SPCG_WIDE_MIN overrides the threshold (mean dependencies per row)
+        const char* wm = getenv("SPCG_WIDE_MIN");
+        const double wmin = wm ? atof(wm) : (double)SPCG_WCAP;
         T.wide = (strategy == SPCG_SPTRSV_LEVEL || strategy == SPCG_SPTRSV_SYNCFREE) && n > 0 &&
-                 (double)deps / (double)n > (double)SPCG_WCAP;
+                 (double)deps / (double)n > wmin;
         if (T.wide) {
             T.wrow.assign(order.begin(), order.end());
             T.wgptr.assign(grp_rows_ptr.begin(), grp_rows_ptr.end());
@@ -683,7 +686,10 @@ void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, 
         partition_rows(F, parts, PT, &out.partition);
         size_t maxsz = 1;
         for (int c = 0; c < parts; ++c) maxsz = std::max(maxsz, PT.rows[c].size());
-        int32_t ring = 1;
+        // >= 16 entries: the ring occupies the front of dynamic shared memory and the
+        // chunk slots behind it need 128-byte alignment (TMA destination, 16-byte header
+        // loads); a 1- or 2-entry ring (n = 1) misaligned them (found by the n = 1 test)
+        int32_t ring = 16;
         while ((size_t)ring < maxsz && ring < ring_max) ring <<= 1;
         out.ring = ring;
         for (int c = 0; c < parts; ++c) out.part_begin[c + 1] = out.part_begin[c] + (int64_t)PT.rows[c].size();

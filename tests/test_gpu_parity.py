@@ -181,3 +181,29 @@ def test_async_concurrent_solves_match_sync():
         assert torch.equal(x, xr)
     with pytest.raises(lib.SpcgError):
         hs[0].solve_wait()                       # nothing in flight
+
+
+@pytest.mark.parametrize("ex", EXECUTORS)
+def test_degenerate_cases(ex):
+    """Edge cases of Algorithm 1 on every executor: b = 0 stops at k = 0
+    with x = 0 (test before the first SpMV, A13); kmax = 0 returns x0 = 0 with
+    NOT_CONVERGED (A14); n = 1 and a diagonal matrix (no off-diagonals: empty L,
+    one wavefront) converge in one iteration with the exact solution."""
+    A = gen.make("poisson2d", 37, 29)
+    h = lib.SPCG(A, sptrsv=ex, parts=5)
+    x, info = h.solve(torch.zeros(A.n, dtype=torch.float64, device="cuda"), eps=1e-8, kmax=100)
+    assert info["iterations"] == 0 and info["status"] == 0 and not torch.any(x != 0)
+    b, _ = gen.rhs(A)
+    x, info = h.solve(_dev(b), eps=1e-8, kmax=0)
+    assert info["iterations"] == 0 and info["status"] == lib.NOT_CONVERGED and not torch.any(x != 0)
+    h.close()
+    for d in (np.array([[3.0]]), np.diag(np.linspace(1.0, 7.0, 5000))):
+        Ad = gen.from_dense(d) if d.shape[0] == 1 else gen.CSR(d.shape[0], np.arange(d.shape[0] + 1, dtype=np.int64),
+                                                               np.arange(d.shape[0], dtype=np.int32), np.diag(d).copy())
+        bd = np.linspace(-1.0, 1.0, Ad.n) if Ad.n > 1 else np.array([1.5])
+        hd = lib.SPCG(Ad, mode="alg2", sptrsv=ex)
+        assert hd.info["levels_L"] == 1
+        xd, info = hd.solve(_dev(bd), eps=1e-12, kmax=10)
+        assert info["iterations"] == 1 and info["status"] == 0
+        assert np.allclose(xd.cpu().numpy(), bd / np.diag(d), rtol=1e-15, atol=0)
+        hd.close()
