@@ -347,6 +347,7 @@ __device__ void phase_spmv(const Params& P, const double* pin, double* wout, dou
     }
 }
 
+constexpr int SF_PF = 4;               // SYNCFREE: dependencies per row read in one batch
 // One slice (<= 32 rows of one wavefront) of a triangular solve, thread per row.
 // Lower (UPPER=false): y_i = r_i - sum_j l_ij y_j   (unit diagonal)
 // Upper (UPPER=true):  z_i = (y_i - sum_j u_ij z_j) / u_ii
@@ -382,7 +383,38 @@ __device__ __forceinline__ void tri_slice(const Params& P, const DevTri& T, int6
         } else {
             acc = in[row];
         }
-        for (int k = 0; k < len; ++k) {
+        int k0 = 0;
+        if (STRAT == ST_SYNCFREE) {
+            // all (index, value) pairs of the row first, then every flag read in one batch:
+            // one memory round trip per slice instead of one per dependency
+            int sx[SF_PF];
+            double vv[SF_PF];
+            uint4 f[SF_PF];
+#pragma unroll
+            for (int k = 0; k < SF_PF; ++k) {
+                sx[k] = k < len ? __ldg(sp + 32 * k) : -1;
+                vv[k] = k < len ? __ldg(vp + 32 * k) : 0.0;
+            }
+#pragma unroll
+            for (int k = 0; k < SF_PF; ++k)
+                if (k < len) {
+                    const uint4* a = mb + (-sx[k] - 1);
+                    asm volatile("ld.volatile.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                                 : "=r"(f[k].x), "=r"(f[k].y), "=r"(f[k].z), "=r"(f[k].w)
+                                 : "l"(a)
+                                 : "memory");
+                }
+#pragma unroll
+            for (int k = 0; k < SF_PF; ++k)
+                if (k < len) {
+                    const double d = (f[k].y == ep && f[k].w == ep)
+                                         ? __longlong_as_double((long long)(((unsigned long long)f[k].z << 32) | f[k].x))
+                                         : ll_wait(mb + (-sx[k] - 1), ep, P.sc);
+                    acc = fma(-vv[k], d, acc);
+                }
+            k0 = SF_PF;
+        }
+        for (int k = k0; k < len; ++k) {
             const int sidx = __ldg(sp + 32 * k);
             const double v = __ldg(vp + 32 * k);
             double d;
