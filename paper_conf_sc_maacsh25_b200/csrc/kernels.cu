@@ -641,7 +641,10 @@ __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const doub
 //                 ahead so only ring gather -> FMA -> store sits on the critical path
 constexpr int PRODUCER_WARP = 0;
 constexpr int POLLER_WARP = 1;
-constexpr int NPOLL = NWARP >= 8 ? 2 : 1;         // poller warps (records alternate)
+#ifndef SPCG_NPOLL
+#define SPCG_NPOLL (SPCG_BLOCK >= 256 ? 2 : 1)
+#endif
+constexpr int NPOLL = SPCG_NPOLL;                 // poller warps (records alternate; 0: the solver polls)
 constexpr int VEC_WARP0 = POLLER_WARP + NPOLL;
 constexpr int NVEC = NWARP - 2 - NPOLL;           // 4 (8 warps) or 1 (4 warps)
 constexpr int SOLVER_WARP0 = VEC_WARP0 + NVEC;
@@ -1282,7 +1285,7 @@ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st, int c0, i
             for (int r = 0; r < nrec; ++r, ++recn) {
                 const Rec R(ch + *(const uint16_t*)(ch + 8 + 2 * r));
                 if (lane == 0 && pw == 0) hbeat(P, 3, ((unsigned long long)(st.k + 1) << 40) | (unsigned long long)recn);
-                if ((int)(recn % NPOLL) != pw || !(R.flags() & REC_FIRST)) continue;
+                if ((int)(recn % (NPOLL > 0 ? NPOLL : 1)) != pw || !(R.flags() & REC_FIRST)) continue;
                 const int2 lw = R.lane(lane);
                 const int ne = lw.x >= 0 ? meta_ne((unsigned)lw.y) : 0;
                 if (!__any_sync(0xffffffffu, ne > 0)) continue;
