@@ -366,6 +366,38 @@ def chain_floor(calib: dict, info: dict, bytes_per_iter: float, peak_gbs: float,
                     "through flags (pipelined), so its true floor lies between the syncthreads and flag rows"}
 
 
+def batch_cpu_baseline(systems, results, budget_s: float = 20.0):
+    """The oracle (single thread) on a bounded sample of C5: the systems in index order
+    until ~budget_s of CPU work, each solved to eps; the batch figure is projected by
+    the GPU iteration counts and the oracle's measured time per iteration per row."""
+    import oracle
+    t_used, rates, done = 0.0, {}, []
+    for s in systems:
+        if t_used > budget_s:
+            break
+        A = gen.make(s.family, *s.params)
+        if A.n > 300000:
+            continue
+        b, _ = gen.rhs(A)
+        L, U, _ = oracle.setup(A, mode="alg2", K=s.K)
+        r = oracle.pcg(A, L, U, b, EPS, 20000)
+        t_used += r["seconds"]
+        rates.setdefault(s.family, []).append(r["seconds"] / max(r["k"] + 1, 1) / A.nnz)
+        done.append(s.index)
+    if not rates:
+        return None
+    # s per (iteration x stored entry of A), per family (ILU(2) factors cost more per entry of A)
+    fam_rate = {f: float(np.median(v)) for f, v in rates.items()}
+    any_rate = float(np.median([x for v in rates.values() for x in v]))
+    fam = {s.index: s.family for s in systems}
+    nnz = {s.index: gen.make(s.family, *s.params).nnz for s in systems}
+    proj = sum(fam_rate.get(fam[r.index], any_rate) * (r.iterations + 1) * nnz[r.index] for r in results) * 1e3
+    return {"value": proj, "unit": "ms", "cores": 1, "kind": "oracle",
+            "sample": f"{len(done)} of {len(systems)} systems solved to eps by the oracle ({t_used:.1f} s); the "
+                      f"batch is projected with the median s per (iteration x nnz(A)) and the GPU iteration "
+                      f"counts, single thread, {_cpu_info()}"}
+
+
 def run_batch(args, ws, rank, local):
     """C5: independent systems spread over the ranks by LPT; no collective on the data path.
 
@@ -447,7 +479,7 @@ def run_batch(args, ws, rank, local):
                              "traffic": None, "kernel": "spcg_pcg_kernel (one launch per system)",
                              "peak_source": peak_src,
                              "achieved_def": "sum over systems of B_iter x iterations / makespan"},
-                "cpu_baseline": None,
+                "cpu_baseline": None if args.no_cpu_baseline else batch_cpu_baseline(systems, allr),
                 "e2e": {"value": e2e_ms, "unit": "ms", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": h2d,
                         "path": "spcg_solve with SPCG_HOST_PTRS per system (wall clock of the rank's loop)"},
                 "gpu_launches": len(systems) * args.steps,
