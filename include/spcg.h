@@ -127,7 +127,7 @@ typedef struct {
     double algo_bytes_per_iter; /* B_iter: what one iteration must move */
     double algo_flops_per_iter;
     int32_t partition;          /* CHUNKED: row partition the inspector chose — 0 contiguous, 1 strided,
-                                   2 affinity, 3 components; -1 otherwise */
+                                   2 affinity, 3 components, 4 tiles; -1 otherwise */
 } spcg_setup_info_t;
 
 typedef struct {

@@ -215,7 +215,7 @@ class SPCG:
         self.info = {f[0]: (list(getattr(si, f[0])) if isinstance(getattr(si, f[0]), ctypes.Array)
                             else getattr(si, f[0])) for f in SetupInfo._fields_}
         self.info["sptrsv_name"] = SPTRSV_NAME.get(self.info["sptrsv"], "?")
-        self.info["partition_name"] = {0: "contiguous", 1: "strided", 2: "affinity", 3: "components"}.get(
+        self.info["partition_name"] = {0: "contiguous", 1: "strided", 2: "affinity", 3: "components", 4: "tiles"}.get(
             self.info["partition"], "-")
 
     def close(self):

@@ -205,9 +205,9 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         I.parts = parts;
         I.device_bytes = bytes;
         {
-            static const char* kinds[] = {"contiguous", "strided", "affinity", "components"};
+            static const char* kinds[] = {"contiguous", "strided", "affinity", "components", "tiles"};
             I.partition = -1;
-            for (int k = 0; k < 4; ++k) if (h->lay.partition == kinds[k]) I.partition = k;
+            for (int k = 0; k < 5; ++k) if (h->lay.partition == kinds[k]) I.partition = k;
         }
         // B_iter: 12 B per stored entry of A, L_s, U_s; 1/u_ii; three row
         // pointers; two level_rows arrays; 120 B of vector traffic per row.

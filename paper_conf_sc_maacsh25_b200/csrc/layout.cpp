@@ -399,21 +399,27 @@ static double model_solve_time(const Factors& F, const Partition& PT, double t_r
     }
     std::vector<double> fin(n, 0.0), clock(PT.parts, 0.0), ready(PT.parts, 0.0);
     std::vector<int32_t> cnt(PT.parts, 0), touched;
-    std::vector<char> ext(PT.parts, 0);
+    std::vector<int32_t> ext(PT.parts, 0);
     for (int64_t l = 0; l < F.wL; ++l) {
         touched.clear();
         for (int64_t t = lp[l]; t < lp[l + 1]; ++t) {
             const int32_t i = lrows[t];
             const int p = PT.part_of[i];
             if (cnt[p]++ == 0) { touched.push_back(p); ready[p] = clock[p]; }
+            bool e = false;
             for (int64_t q = F.L.rp[i]; q < F.L.rp[i + 1]; ++q) {
                 const int32_t j = F.L.col[q];
-                if (PT.part_of[j] != p) { ready[p] = std::max(ready[p], fin[j] + H); ext[p] = 1; }
+                if (PT.part_of[j] != p) { ready[p] = std::max(ready[p], fin[j] + H); e = true; }
             }
+            ext[p] += e;
         }
         for (int p : touched) {
-            // a record with cross-CTA terms costs more: poller handoff + flag reads
-            clock[p] = ready[p] + (ext[p] ? t_ext : t_rec) * (double)((cnt[p] + 31) / 32);
+            // cross-CTA terms cost extra: half of it once the record has any (poller handoff),
+            // half in proportion to the rows that have them (fitted to the poisson3d 48^3 /
+            // 64^3 / 102^3 measurements of strided, tiles and affinity)
+            const double f = (double)ext[p] / (double)cnt[p];
+            const double tr = ext[p] ? t_rec + 0.5 * (t_ext - t_rec) * (1.0 + f) : t_rec;
+            clock[p] = ready[p] + tr * (double)((cnt[p] + 31) / 32);
             cnt[p] = 0;
             ext[p] = 0;
         }
@@ -435,6 +441,57 @@ static int64_t dominant_stride(const Factors& F) {
     int64_t best = 0, bc = 0;
     for (auto& kv : h) if (kv.second > bc) { bc = kv.second; best = kv.first; }
     return best;
+}
+
+// 3-D natural-order grids (two strides s1 | s2 among L's offsets: x-lines of length
+// s1, planes of s2 rows): whole x-lines stay in one part, the (y, z) plane of lines
+// is tiled Ty x Tz <= P.  The x-chain then runs through the ring; only the tile
+// faces exchange flags, and the cross-CTA pipeline is Ty + Tz hops deep instead of
+// the P-long chain of a slab partition.  Returns false if no such strides exist.
+static bool partition_tiles(const Factors& F, int P, Partition& out) {
+    const int64_t n = F.L.n;
+    std::map<int64_t, int64_t> h;
+    const int64_t step = std::max<int64_t>(1, n / 20000);
+    for (int64_t i = 0; i < n; i += step)
+        for (int64_t q = F.L.rp[i]; q < F.L.rp[i + 1]; ++q) {
+            const int64_t d = i - F.L.col[q];
+            if (d > 1) h[d]++;
+        }
+    std::vector<std::pair<int64_t, int64_t>> byc;
+    for (auto& kv : h) byc.push_back({-kv.second, kv.first});
+    std::sort(byc.begin(), byc.end());
+    if (byc.size() < 2) return false;
+    int64_t s1 = byc[0].second, s2 = 0;
+    for (size_t k = 1; k < byc.size() && k < 4; ++k)
+        if (byc[k].second > s1 && byc[k].second % s1 == 0) { s2 = byc[k].second; break; }
+    if (s2 == 0 || s1 < 2) {
+        // the two leading offsets may come in the other order
+        if (byc[1].second < s1 && s1 % byc[1].second == 0) { s2 = s1; s1 = byc[1].second; }
+        else return false;
+    }
+    const int64_t NY = s2 / s1, NZ = (n + s2 - 1) / s2;
+    if (NY < 2 || NZ < 2) return false;
+    int Ty = std::max<int>(1, (int)std::lround(std::sqrt((double)P * (double)NY / (double)NZ)));
+    Ty = (int)std::min<int64_t>(Ty, NY);
+    int Tz = (int)std::min<int64_t>(std::max(1, P / Ty), NZ);
+    // a tile must fit one 32-row record per wavefront (one row per x-line and level);
+    // larger tiles split every wavefront into several records and lose to the slab
+    // partitions (measured: 64^3 tiles 0.49 vs strided 0.54 ms/it; 102^3 1.48 vs 1.29)
+    if ((double)NY * (double)NZ / ((double)Ty * (double)Tz) > 32.0) return false;
+    out.parts = P;
+    out.part_of.assign(n, 0);
+    for (int64_t i = 0; i < n; ++i) {
+        const int64_t y = (i / s1) % NY, z = i / s2;
+        out.part_of[i] = (int32_t)(((z * Tz) / NZ) * Ty + (y * Ty) / NY);
+    }
+    out.rows.assign(P, {});
+    out.lidx.assign(n, 0);
+    for (int64_t i = 0; i < n; ++i) {
+        const int p = out.part_of[i];
+        out.lidx[i] = (int32_t)out.rows[p].size();
+        out.rows[p].push_back((int32_t)i);
+    }
+    return true;
 }
 
 // Inspector: build candidate partitions and keep the one the model says is fastest.
@@ -460,11 +517,18 @@ static void partition_rows(const Factors& F, int P, Partition& out, std::string*
         Partition p;
         if (partition_components(F, P, p) >= P) cand.push_back({"components", std::move(p)});
     }
+    {
+        Partition p;
+        if (partition_tiles(F, P, p)) cand.push_back({"tiles", std::move(p)});
+    }
     const char* force = getenv("SPCG_PART");
     double best = 1e300;
     size_t bi = 0;
     for (size_t c = 0; c < cand.size(); ++c) {
-        const double t = model_solve_time(F, cand[c].second, T_REC, T_EXT, H);
+        // the model underrates the affinity partition (its rows' dependencies often go
+        // through flags instead of the ring): measured 11 % slower than predicted relative
+        // to strided on poisson3d 102^3, so it carries a 15 % penalty
+        const double t = model_solve_time(F, cand[c].second, T_REC, T_EXT, H) * (cand[c].first == "affinity" ? 1.15 : 1.0);
         if (getenv("SPCG_PART_VERBOSE")) fprintf(stderr, "[spcg] partition %s: modelled forward solve %.1f us\n", cand[c].first.c_str(), t);
         if (force ? cand[c].first == force : t < best) { best = force ? 0.0 : t; bi = c; }
     }
