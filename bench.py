@@ -303,6 +303,11 @@ def main():
     s_gbs = s_bi * s["k"] / (s_ms * 1e-3) / 1e9
     p_gbs = p_bi * p["k"] / (p_ms * 1e-3) / 1e9
     traffic = _ncu_traffic(name, "spcg", s["k"])
+    l2_hit = None
+    try:
+        l2_hit = json.load(open(os.path.join(ROOT, "profiles", "ncu_summary.json")))[name]["spcg"].get("l2_hit_pct")
+    except Exception:
+        pass
     cpu = None
     if not args.no_cpu_baseline:
         o = run_oracle(name, A, b, 2, 0, budget_s=20.0, k_hint={"alg2": s["k"], "none": p["k"]})
@@ -333,7 +338,11 @@ def main():
         "roofline": {"bound": "hbm", "achieved": s_gbs, "peak": peak, "unit": "GB/s", "frac": s_gbs / peak,
                      "traffic": traffic, "kernel": "spcg_pcg_kernel (persistent, whole Alg. 1)",
                      "peak_source": peak_src,
-                     "achieved_def": "B_iter (DESIGN.md §4) x iterations / CUDA-event time of the launch"},
+                     "achieved_def": "B_iter (DESIGN.md §4) x iterations / CUDA-event time of the launch",
+                     "l2_hit_pct": l2_hit,
+                     "note": ("working set L2-resident (B_iter < 126 MB L2; ncu DRAM traffic << algorithmic): "
+                              "the HBM roofline is not the binding one; the chain floor is (chain_floor)"
+                              if s_bi < 100e6 else "the wavefront chain binds before HBM (chain_floor)")},
         "cpu_baseline": cpu,
         "chain_floor": chain_floor(calib, si, s_bi, peak, s_ms / max(s["k"], 1)),
         "e2e": {"value": s_e2e, "unit": "ms", "h2d_bytes_per_step": 8 * A.n, "d2h_bytes_per_step": 8 * A.n,
