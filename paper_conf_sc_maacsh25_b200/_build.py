@@ -52,7 +52,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     for cpp in sorted(glob.glob(os.path.join(CSRC, "*.cpp"))):
         o = os.path.join(bdir, os.path.basename(cpp) + ".o")
         cmd = ["g++", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-fPIC", "-std=c++17",
-               "-I", os.path.join(ROOT, "include"), "-I", "/usr/local/cuda/include", "-c", cpp, "-o", o]
+               "-I", os.path.join(ROOT, "include"), "-I", "/usr/local/cuda/include", *defines, "-c", cpp, "-o", o]
         subprocess.check_call(cmd)
         objs.append(o)
     tmp = lib + ".tmp"

@@ -99,7 +99,12 @@ constexpr int SPCG_CHUNK_BYTES = 4096;
 constexpr int SPCG_NCHUNK = SPCG_NCHUNK_SLOTS;   // chunk ring slots in shared memory (kernel side)
 constexpr int SPCG_MAXREC = 8;          // records per chunk (side-data slots)
 constexpr int SPCG_WCAP = 8;            // entry columns per record
-constexpr int SPCG_NSOLVER = 1;         // solver warps per CTA (one software-pipelined chain)
+#ifndef SPCG_NSOLVER_WARPS
+#define SPCG_NSOLVER_WARPS 1
+#endif
+// solver warps per CTA: the slices of a part's stream are dealt round-robin to them
+// and a shared-memory chain counter orders their ring accesses
+constexpr int SPCG_NSOLVER = SPCG_NSOLVER_WARPS;
 constexpr int SPCG_REC_HDR = 272;       // 16 B header + 32 x {int32 row, uint32 meta}
 constexpr int SPCG_CHUNK_HDR = 32;      // u16 nrec, u16 -, u32 used, u16 rec_off[8], pad
 enum { REC_FIRST = 1, REC_LAST = 2, REC_SYNC = 4, REC_UPPER = 8, REC_EXT = 16, REC_WIDE = 32 };

@@ -642,11 +642,12 @@ __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const doub
 constexpr int PRODUCER_WARP = 0;
 constexpr int POLLER_WARP = 1;
 #ifndef SPCG_NPOLL
-#define SPCG_NPOLL (SPCG_BLOCK >= 256 ? 2 : 1)
+#define SPCG_NPOLL (SPCG_BLOCK >= 256 && SPCG_NSOLVER_WARPS == 1 ? 2 : 1)
 #endif
 constexpr int NPOLL = SPCG_NPOLL;                 // poller warps (records alternate; 0: the solver polls)
 constexpr int VEC_WARP0 = POLLER_WARP + NPOLL;
-constexpr int NVEC = NWARP - 2 - NPOLL;           // 4 (8 warps) or 1 (4 warps)
+constexpr int NVEC = NWARP - 1 - NPOLL - SPCG_NSOLVER;   // 4 (8 warps, 1 solver) ...
+static_assert(NVEC >= 1, "at least one vector warp");
 constexpr int SOLVER_WARP0 = VEC_WARP0 + NVEC;
 static_assert(SOLVER_WARP0 + SPCG_NSOLVER == NWARP, "warp roles must fill the CTA");
 #ifndef SPCG_SOLVER_TREE
@@ -672,7 +673,7 @@ constexpr int SIDE_BYTES = 3 * 256 + 16;          // vec[32], aux[32], ext[32], 
 constexpr size_t CH_RING_BYTES = (size_t)SPCG_NCHUNK * SPCG_CHUNK_BYTES;
 constexpr size_t CH_SIDE_BYTES = (size_t)SPCG_NCHUNK * SPCG_MAXREC * SIDE_BYTES;
 constexpr size_t CH_BAR_BYTES = 512;
-static_assert((3 * SPCG_NCHUNK + 1 + SPCG_NSOLVER + 1) <= 32 && 256 + 2 * NVEC * VLIST <= CH_BAR_BYTES,
+static_assert((3 * SPCG_NCHUNK + 1 + SPCG_NSOLVER + 1) <= 31 && 256 + 2 * NVEC * VLIST <= CH_BAR_BYTES,
               "barrier block layout");
 
 __host__ __device__ constexpr size_t chunked_smem_bytes(int ring) {
@@ -689,6 +690,7 @@ struct ChunkSmem {
     uint64_t* ldone;       // solvers finished the L section
     volatile long long* progress;   // [NSOLVER] record index each solver warp is at
     uint16_t* vlist;       // [NVEC][VLIST] per vector warp: (slot, record) of its records in a group
+    volatile unsigned* chain;   // multi-solver: slices of this phase completed (ring accesses ordered by it)
 };
 
 struct PipeState {         // identical sequence in every role
@@ -772,6 +774,7 @@ __device__ ChunkSmem chunk_smem(double* dyn, int ring) {
     S.ldone = bars + 3 * SPCG_NCHUNK;
     S.progress = (volatile long long*)(bars + 3 * SPCG_NCHUNK + 1);
     S.vlist = (uint16_t*)(bars + 32);
+    S.chain = (volatile unsigned*)(bars + 31);
     return S;
 }
 
@@ -784,6 +787,7 @@ __device__ void chunk_init(const ChunkSmem& S) {
         }
         mbar_init(S.ldone, SPCG_NSOLVER);
         for (int i = 0; i < SPCG_NSOLVER; ++i) S.progress[i] = -1;
+        *S.chain = 0u;
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -1129,6 +1133,64 @@ __device__ __forceinline__ void solver_section(const SolveCtx& C, const ChunkSme
     }
 }
 
+// Several solver warps (SPCG_NSOLVER > 1): the slices of the part's stream are
+// dealt round-robin to them (record header `warp`, layout.cpp); every solver warp
+// walks all records to number the slices of this phase, prepares its own records
+// ahead, then waits until the chain counter says every earlier slice is done,
+// runs the record (ring gathers -> FMAs -> ring / global stores) and, after the
+// slice's last record, publishes chain = slice + 1 (release fence, then a
+// volatile store).  The ring is therefore read and written in exactly the
+// sequential slice order the layout's ring analysis assumes, while each warp's
+// instruction stream carries only 1/NSOLVER of the records.
+__device__ __forceinline__ bool chain_wait(const ChunkSmem& S, unsigned s, Scal* sc) {
+    const int lane = threadIdx.x & 31;
+    unsigned it = 0;
+    const long long t0 = clock64();
+    for (;;) {
+        const unsigned c = __shfl_sync(0xffffffffu, lane == 0 ? *S.chain : 0u, 0);
+        if ((int)(c - s) >= 0) return true;
+        if ((++it & 1023) == 0) {
+            const bool late = __shfl_sync(0xffffffffu, clock64() - t0 > SPIN_TIMEOUT_CYC, 0);
+            if (late && lane == 0) atomicExch(&sc->abort, 1);
+            if (late || aborted(sc)) return false;
+        }
+    }
+}
+
+template <bool UPPER, bool PRO>
+__device__ __noinline__ void solver_section_multi(const SolveCtx& C, const ChunkSmem& S, unsigned q0, int ib, int ie,
+                                                  unsigned& lseq, double& rz, int sw, long long recn) {
+    const int lane = threadIdx.x & 31;
+    double acc_carry = 0.0;
+    for (int i = ib; i < ie; ++i) {
+        const unsigned q = q0 + i;
+        const int slot = q % SPCG_NCHUNK;
+        if (!warp_ok(mbar_wait(&S.vfull[slot], (q / SPCG_NCHUNK) & 1, C.sc))) return;
+        const uint8_t* ch = S.chunks + (size_t)slot * SPCG_CHUNK_BYTES;
+        const int nrec = *(const uint16_t*)ch;
+        if (sw == 0 && lane == 0) S.progress[0] = recn;
+        recn += nrec;
+        for (int r = 0; r < nrec; ++r) {
+            const uint8_t* p = ch + *(const uint16_t*)(ch + 8 + 2 * r);
+            const int fl = (int)(*(const uint32_t*)p >> 16);
+            const int owner = p[4];
+            const unsigned sl = (fl & REC_FIRST) ? lseq++ : lseq - 1;   // slice of this record
+            if (owner != sw) continue;
+            Prep X;
+            prep_record<UPPER>(X, S, ch, slot, r, lane);
+            if ((fl & REC_FIRST) && !chain_wait(S, sl, C.sc)) return;
+            solve_record<UPPER, PRO>(C, X, slot, lane, acc_carry, rz);
+            if (fl & REC_LAST) {
+                fence_acq_rel_cta();            // this warp's ring stores before the counter
+                __syncwarp();
+                if (lane == 0) *S.chain = sl + 1;
+            }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&S.empty[slot]);
+    }
+}
+
 // One triangular-solve phase of a part: chunks [c0, c1) of its stream (L section,
 // U section or both).  All threads of the CTA call it.
 #if SPCG_PHASE_NOINLINE
@@ -1323,11 +1385,29 @@ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st, int c0, i
             if (lane == 0) mbar_arrive(&S.empty[slot]);
         }
     } else {
-        // ---------------- solver warp (one per CTA)
+        // ---------------- solver warp(s)
         const int ncL = (c0 < cu) ? min(cu, c1) - c0 : 0;       // chunks of the L section
         if (lane == 0) trace_mark(P, st.k, 8 + 4 * blockIdx.x + 0);
         SolveCtx C{S.yring, &S, y, nullptr, P.p, P.mbL, P.sc, ep, pb, mask};
-        if (ncL > 0) {
+        if (SPCG_NSOLVER > 1) {
+            const int sw = warp - SOLVER_WARP0;
+            unsigned lseq = 0;
+            if (ncL > 0) {
+                double dummy = 0.0;
+                solver_section_multi<false, false>(C, S, q0, 0, ncL, lseq, dummy, sw, rec0);
+                __syncwarp();
+                if (lane == 0 && c1 > cu) mbar_arrive(S.ldone);
+            }
+            if (ncL < nch) {
+                long long n = 0;
+                for (int t = 0; t < ncL; ++t) n += *(const uint16_t*)(P.stream + (size_t)(c0 + t) * SPCG_CHUNK_BYTES);
+                C.out = z;
+                C.rdot = rdot;
+                C.mb = P.mbU;
+                if (kind == K_PRO) solver_section_multi<true, true>(C, S, q0, ncL, nch, lseq, rz, sw, rec0 + n);
+                else solver_section_multi<true, false>(C, S, q0, ncL, nch, lseq, rz, sw, rec0 + n);
+            }
+        } else if (ncL > 0) {
             double dummy = 0.0;
             solver_section<false, false>(C, S, q0, 0, ncL, rec0, dummy, P, st.k);
             __syncwarp();
@@ -1336,7 +1416,7 @@ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st, int c0, i
                 trace_mark(P, st.k, 8 + 4 * blockIdx.x + 1);
             }
         }
-        if (ncL < nch) {
+        if (SPCG_NSOLVER == 1 && ncL < nch) {
             long long n = 0;                                        // U records continue the numbering
             for (int t = 0; t < ncL; ++t) n += *(const uint16_t*)(P.stream + (size_t)(c0 + t) * SPCG_CHUNK_BYTES);
             C.out = z;
@@ -1360,8 +1440,10 @@ void chunked_phase(const Params& P, const ChunkSmem& S, PipeState& st, int c0, i
     __syncthreads();
     st.rec = S.progress[SPCG_NSOLVER];
     if (threadIdx.x == 0) trace_mark(P, st.k, 8 + 4 * blockIdx.x + 3);
-    if (threadIdx.x == 0)
+    if (threadIdx.x == 0) {
         for (int i = 0; i < SPCG_NSOLVER; ++i) S.progress[i] = st.rec - 1;
+        *S.chain = 0u;                       // the next phase numbers its slices from 0
+    }
     __syncthreads();
 }
 

@@ -613,7 +613,7 @@ void put(uint8_t* base, size_t off, T v) { std::memcpy(base + off, &v, sizeof(T)
 static void emit_section(StreamWriter& W, const Csr& M, bool upper, const std::vector<int32_t>& lev,
                          const std::vector<int32_t>& prow, const Partition& PT, const std::vector<int32_t>& step_of,
                          const std::vector<int32_t>& next_writer, const std::vector<uint8_t>& publish, int32_t ring,
-                         bool sync_first) {
+                         bool sync_first, int64_t& seq) {
     if (prow.empty()) return;
     auto dep_begin = [&](int64_t i) { return upper ? M.rp[i] + 1 : M.rp[i]; };
     // rows of the part grouped by level (ascending), rows ascending inside a level
@@ -651,7 +651,7 @@ static void emit_section(StreamWriter& W, const Csr& M, bool upper, const std::v
                 for (int32_t sidx : esrc[l]) ne_tot[l] += sidx < 0;
                 wmax = std::max<int>(wmax, (int)esrc[l].size());
             }
-            const int warp = sl % SPCG_NSOLVER;
+            const int warp = (int)(seq++ % SPCG_NSOLVER);   // slices of the part's stream, round-robin
             int k0 = 0;
             do {
                 const int wp = std::min(SPCG_WCAP, wmax - k0);
@@ -730,10 +730,11 @@ static void build_chunk_stream(const Factors& F, const Partition& PT, int32_t ri
     for (int c = 0; c < parts; ++c) {
         W.new_chunk();
         S.part_chunk[c] = (int32_t)W.cur;
-        emit_section(W, F.L, false, F.levL, PT.rows[c], PT, stepL, nwL, pubL, ring, false);
+        int64_t seq = 0;                     // slice sequence of this part (L then U section)
+        emit_section(W, F.L, false, F.levL, PT.rows[c], PT, stepL, nwL, pubL, ring, false, seq);
         W.new_chunk();                     // U section starts on a chunk boundary
         S.part_uchunk[c] = (int32_t)W.cur;
-        emit_section(W, F.U, true, F.levU, PT.rows[c], PT, stepU, nwU, pubU, ring, true);
+        emit_section(W, F.U, true, F.levU, PT.rows[c], PT, stepU, nwU, pubU, ring, true, seq);
     }
     W.finish();
     S.part_chunk[parts] = (int32_t)(S.bytes.size() / SPCG_CHUNK_BYTES);
