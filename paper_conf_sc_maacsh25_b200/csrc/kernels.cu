@@ -1179,6 +1179,32 @@ __device__ __noinline__ void solver_section_multi(const SolveCtx& C, const Chunk
             Prep X;
             prep_record<UPPER>(X, S, ch, slot, r, lane);
             if ((fl & REC_FIRST) && !chain_wait(S, sl, C.sc)) return;
+            if ((X.fl & (REC_FIRST | REC_LAST | REC_WIDE | REC_EXT)) == (REC_FIRST | REC_LAST)) {
+                // fast path with the chain handoff before the global stores: ring store,
+                // fence, counter, and only then out[] / p / the ready flag (a fence after
+                // the global stores would wait for them)
+                double d[WP];
+#pragma unroll
+                for (int k = 0; k < WP; ++k) d[k] = C.yring[X.sidx[k]];
+                double acc = X.vec;
+#pragma unroll
+                for (int k = 0; k < WP; ++k) acc = fma(-X.v[k], d[k], acc);
+                if (UPPER) acc *= X.dinv;
+                if (X.row >= 0) C.yring[X.meta >> 17] = acc;
+                fence_acq_rel_cta();
+                __syncwarp();
+                if (lane == 0) *S.chain = sl + 1;
+                if (X.row >= 0) {
+                    if (UPPER) {
+                        rz = fma(X.aux, acc, rz);
+                        if (PRO) C.pvec[X.row] = acc;
+                    }
+                    C.out[X.row] = acc;
+                    if (meta_pub(X.meta)) ll_store((uint4*)C.mb + X.row, acc, C.ep);
+                }
+                acc_carry = acc;
+                continue;
+            }
             solve_record<UPPER, PRO>(C, X, slot, lane, acc_carry, rz);
             if (fl & REC_LAST) {
                 fence_acq_rel_cta();            // this warp's ring stores before the counter
