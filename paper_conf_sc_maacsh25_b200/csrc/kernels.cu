@@ -661,7 +661,10 @@ static_assert(SOLVER_WARP0 + SPCG_NSOLVER == NWARP, "warp roles must fill the CT
                                    // live in local memory: 1.5x slower per iteration, measured)
 #endif
 constexpr int kSolverUnroll = SPCG_SOLVER_UNROLL;
-constexpr int POLL_AHEAD = 8;                     // records
+#ifndef SPCG_POLL_AHEAD
+#define SPCG_POLL_AHEAD 8
+#endif
+constexpr int POLL_AHEAD = SPCG_POLL_AHEAD;       // records
 #ifndef SPCG_VGROUP
 #define SPCG_VGROUP 4
 #endif
