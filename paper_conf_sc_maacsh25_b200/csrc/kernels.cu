@@ -548,33 +548,55 @@ __device__ void tri_syncfree_wide(const Params& P, const DevTri& T, int kind, co
                                   const double* rdot, uint4* mb, unsigned ep, double alpha, double& acc_dot) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int64_t W = (int64_t)gridDim.x * NWARP;
-    for (int64_t q = (int64_t)blockIdx.x * NWARP + warp; q < P.n; q += W) {
-        const int row = __ldg(T.wrow + q);
-        const int64_t e0 = __ldg(T.wptr + q), e1 = __ldg(T.wptr + q + 1);
-        double r0 = 0.0, w0 = 0.0, x0 = 0.0, p0v = 0.0, a0 = 0.0, dv = 1.0;
-        if (lane == 0) {
-            if (!UPPER) {
-                if (kind == K_ITER) { r0 = __ldcg(P.r + row); w0 = __ldcg(P.w + row); x0 = __ldcg(P.x + row); p0v = __ldcg(P.p + row); }
-                else r0 = __ldcg(in + row);
-            } else {
-                r0 = __ldcg(in + row);
-                if (rdot) a0 = __ldcg(rdot + row);
-                dv = __ldg(T.wdinv + q);
-            }
-        }
-        // all of this lane's (index, value) pairs first, then the flag waits
+    // the warp's NEXT row (q + W) is loaded while it waits on the flags of the current
+    // one: index/value pairs and the row's own operands do not depend on any flag
+    struct RowOps {
+        int row;
+        int64_t e0, e1;
         int c[WPF];
         double v[WPF];
+        double r0, w0, x0, p0v, a0, dv;
+    };
+    auto load = [&](int64_t q, RowOps& o) {
+        o.row = __ldg(T.wrow + q);
+        o.e0 = __ldg(T.wptr + q);
+        o.e1 = __ldg(T.wptr + q + 1);
+        o.r0 = o.w0 = o.x0 = o.p0v = o.a0 = 0.0;
+        o.dv = 1.0;
+        if (lane == 0) {
+            if (!UPPER) {
+                if (kind == K_ITER) {
+                    o.r0 = __ldcg(P.r + o.row); o.w0 = __ldcg(P.w + o.row);
+                    o.x0 = __ldcg(P.x + o.row); o.p0v = __ldcg(P.p + o.row);
+                } else {
+                    o.r0 = __ldcg(in + o.row);
+                }
+            } else {
+                o.r0 = __ldcg(in + o.row);
+                if (rdot) o.a0 = __ldcg(rdot + o.row);
+                o.dv = __ldg(T.wdinv + q);
+            }
+        }
 #pragma unroll
         for (int u = 0; u < WPF; ++u) {
-            const int64_t e = e0 + lane + 32 * u;
-            c[u] = e < e1 ? __ldg(T.wcol + e) : -1;
-            v[u] = e < e1 ? __ldg(T.wval + e) : 0.0;
+            const int64_t e = o.e0 + lane + 32 * u;
+            o.c[u] = e < o.e1 ? __ldg(T.wcol + e) : -1;
+            o.v[u] = e < o.e1 ? __ldg(T.wval + e) : 0.0;
         }
+    };
+    RowOps nxt;
+    int64_t q = (int64_t)blockIdx.x * NWARP + warp;
+    if (q < P.n) load(q, nxt);
+    for (; q < P.n; q += W) {
+        const RowOps cur = nxt;
+        if (q + W < P.n) load(q + W, nxt);
+        const int row = cur.row;
+        const int64_t e0 = cur.e0, e1 = cur.e1;
+        const double r0 = cur.r0, w0 = cur.w0, x0 = cur.x0, p0v = cur.p0v, a0 = cur.a0, dv = cur.dv;
         double part = 0.0;
 #pragma unroll
         for (int u = 0; u < WPF; ++u)
-            if (c[u] >= 0) part = fma(v[u], ll_wait(mb + c[u], ep, P.sc), part);
+            if (cur.c[u] >= 0) part = fma(cur.v[u], ll_wait(mb + cur.c[u], ep, P.sc), part);
         for (int64_t e = e0 + lane + 32 * WPF; e < e1; e += 32)
             part = fma(__ldg(T.wval + e), ll_wait(mb + __ldg(T.wcol + e), ep, P.sc), part);
         part = warp_sum(part);
