@@ -45,7 +45,7 @@ constexpr int BLOCK = SPCG_BLOCK;
 #define SPCG_CTAS_PER_SM (SPCG_BLOCK == 128 ? 2 : 1)   // persistent CTAs per SM (independent chains per SM)
 #endif
 #ifndef SPCG_RING_MAX
-#define SPCG_RING_MAX (SPCG_CTAS_PER_SM > 1 ? 4096 : 16384)   // shared-memory ring entries (power of two)
+#define SPCG_RING_MAX (SPCG_CTAS_PER_SM > 1 ? 4096 : 8192)   // shared-memory ring entries (power of two)
 #endif
 constexpr int NWARP = BLOCK / 32;
 constexpr long long SPIN_TIMEOUT_CYC = 8ll * 1000 * 1000 * 1000;            // ~4 s of SM cycles: abort, never hang

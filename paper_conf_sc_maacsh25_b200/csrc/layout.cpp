@@ -749,13 +749,23 @@ void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, 
     if (strategy == SPCG_SPTRSV_CHUNKED) {
         Partition PT;
         partition_rows(F, parts, PT, &out.partition);
-        size_t maxsz = 1;
-        for (int c = 0; c < parts; ++c) maxsz = std::max(maxsz, PT.rows[c].size());
+        // ring size: enough for the longest intra-part dependency distance in part-local
+        // row numbering (slot = lidx & (ring - 1)), not the part size — a small ring leaves
+        // shared memory to the L1 carve-out (layered 4096^2 SPCG: 8192 -> 64 entries).
+        // Anything the ring cannot hold safely goes through the flags (ring analysis).
+        int64_t maxdist = 1;
+        for (const Csr* M : {&F.L, &F.U})
+            for (int64_t i = 0; i < n; ++i)
+                for (int64_t q = M->rp[i]; q < M->rp[i + 1]; ++q) {
+                    const int32_t j = M->col[q];
+                    if (j != i && PT.part_of[j] == PT.part_of[i])
+                        maxdist = std::max<int64_t>(maxdist, std::llabs((int64_t)PT.lidx[i] - PT.lidx[j]));
+                }
         // >= 16 entries: the ring occupies the front of dynamic shared memory and the
         // chunk slots behind it need 128-byte alignment (TMA destination, 16-byte header
         // loads); a 1- or 2-entry ring (n = 1) misaligned them (found by the n = 1 test)
         int32_t ring = 16;
-        while ((size_t)ring < maxsz && ring < ring_max) ring <<= 1;
+        while ((int64_t)ring <= 2 * maxdist && ring < ring_max) ring <<= 1;
         out.ring = ring;
         for (int c = 0; c < parts; ++c) out.part_begin[c + 1] = out.part_begin[c] + (int64_t)PT.rows[c].size();
         build_chunk_stream(F, PT, ring, out.S);

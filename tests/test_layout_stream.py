@@ -24,11 +24,10 @@ import pytest
 import gen
 import paper_conf_sc_maacsh25_b200 as lib
 
-CHUNK = 4096
 REC_FIRST, REC_LAST, REC_UPPER, REC_EXT, REC_WIDE = 1, 2, 8, 16, 32
 
 
-def _records(stream, c0, c1):
+def _records(stream, c0, c1, CHUNK):
     for c in range(c0, c1):
         ch = stream[c * CHUNK:(c + 1) * CHUNK]
         nrec = int(np.frombuffer(ch[:2].tobytes(), np.uint16)[0])
@@ -67,6 +66,8 @@ def test_record_stream_covers_factors(fam, params, K, parts, part, monkeypatch):
     Lrp, Lcol, Lval = h.export("l_rowptr"), h.export("l_col"), h.export("l_val")
     Urp, Ucol, Uval = h.export("u_rowptr"), h.export("u_col"), h.export("u_val")
     levL, levU = h.export("level_l"), h.export("level_u")
+    chunk = len(stream) // int(pch[-1])             # bytes per chunk (a build constant)
+    assert chunk % 1024 == 0 and chunk * int(pch[-1]) == len(stream)
     n = A.n
     seen = {"L": np.zeros(n, np.int32), "U": np.zeros(n, np.int32)}
     for c in range(parts):
@@ -76,7 +77,7 @@ def test_record_stream_covers_factors(fam, params, K, parts, part, monkeypatch):
             rp, col, val = (Urp, Ucol, Uval) if upper else (Lrp, Lcol, Lval)
             rows_part, last_level = [], -1
             entries = {}                                    # row -> list of (src, val)
-            for w, fl, lanes, src, vv, dinv in _records(stream, c0, c1):
+            for w, fl, lanes, src, vv, dinv in _records(stream, c0, c1, chunk):
                 assert bool(fl & REC_UPPER) == upper
                 for l in range(32):
                     r, meta = int(lanes[l, 0]), int(lanes[l, 1]) & 0xFFFFFFFF
