@@ -764,8 +764,27 @@ void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, 
         // >= 16 entries: the ring occupies the front of dynamic shared memory and the
         // chunk slots behind it need 128-byte alignment (TMA destination, 16-byte header
         // loads); a 1- or 2-entry ring (n = 1) misaligned them (found by the n = 1 test)
-        int32_t ring = 16;
-        while ((int64_t)ring <= 2 * maxdist && ring < ring_max) ring <<= 1;
+        int32_t small = 16;
+        while ((int64_t)small <= 2 * maxdist && small < ring_max) small <<= 1;
+        // rows run in wavefront order, not in lidx order, so a short distance does not
+        // make a small ring safe: keep it only if it sends no more dependencies through
+        // the flags than the largest ring does (ring_analysis decides entry by entry)
+        auto unsafe = [&](int32_t R) {
+            int64_t cnt = 0;
+            std::vector<int32_t> st, nw;
+            for (int f = 0; f < 2; ++f) {
+                const Csr& M = f ? F.U : F.L;
+                ring_analysis(PT, f ? F.levU : F.levL, R, st, nw);
+                for (int64_t i = 0; i < n; ++i)
+                    for (int64_t q = M.rp[i]; q < M.rp[i + 1]; ++q) {
+                        const int32_t j = M.col[q];
+                        if (j != i && PT.part_of[j] == PT.part_of[i] && !(nw[j] > st[i])) ++cnt;
+                    }
+            }
+            return cnt;
+        };
+        int32_t ring = ring_max;
+        if (small < ring_max && unsafe(small) <= unsafe(ring_max)) ring = small;
         out.ring = ring;
         for (int c = 0; c < parts; ++c) out.part_begin[c + 1] = out.part_begin[c] + (int64_t)PT.rows[c].size();
         build_chunk_stream(F, PT, ring, out.S);
