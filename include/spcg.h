@@ -92,9 +92,12 @@ enum {
     SPCG_SPTRSV_AUTO = 0,
     SPCG_SPTRSV_LEVEL = 1,      /* level-scheduled: one grid barrier per wavefront */
     SPCG_SPTRSV_SYNCFREE = 2,   /* per-row ready flags, no level barriers */
-    SPCG_SPTRSV_CHUNKED = 3     /* rows partitioned into contiguous per-CTA chunks; intra-chunk
+    SPCG_SPTRSV_CHUNKED = 3,    /* rows partitioned into contiguous per-CTA chunks; intra-chunk
                                    dependencies through shared memory, cross-chunk through flags */
+    SPCG_SPTRSV_RESIDENT = 4    /* small systems (n <= SPCG_RESIDENT_MAX_N): one CTA holds every
+                                   vector in shared memory; level-scheduled with CTA barriers */
 };
+#define SPCG_RESIDENT_MAX_N 4096
 
 typedef struct {
     int32_t device;             /* CUDA ordinal; -1 = host analysis only (export works, solve does not) */

@@ -27,7 +27,8 @@ ERR_INVALID_ARG, ERR_BAD_MATRIX, ERR_ZERO_PIVOT, ERR_BREAKDOWN = -1, -2, -3, -4
 ERR_OOM, ERR_CUDA, ERR_INTERNAL, ERR_NO_DEVICE = -5, -6, -7, -8
 
 DROP_NONE, DROP_FIXED, DROP_WAVEFRONT_AWARE = 0, 1, 2
-SPTRSV = {"auto": 0, "level": 1, "syncfree": 2, "chunked": 3}
+SPTRSV = {"auto": 0, "level": 1, "syncfree": 2, "chunked": 3, "resident": 4}
+RESIDENT_MAX_N = 4096          # include/spcg.h SPCG_RESIDENT_MAX_N
 SPTRSV_NAME = {v: k for k, v in SPTRSV.items()}
 USE_X0, HOST_PTRS = 0x1, 0x2
 

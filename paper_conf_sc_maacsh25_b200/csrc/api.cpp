@@ -158,11 +158,25 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         if (strategy == SPCG_SPTRSV_AUTO) {
             const double wl = h->n > 0 ? (double)h->F.L.nnz() / (double)h->n : 0.0;
             strategy = (h->identity || wl <= (double)SPCG_WCAP) ? SPCG_SPTRSV_CHUNKED : SPCG_SPTRSV_SYNCFREE;
+            // Small systems with >= 32 rows per wavefront on average: the one-CTA resident
+            // executor (vectors in shared memory, CTA barriers) beats the chunked pipeline
+            // (measured per iteration: 16^3 Poisson 129 -> 63 us, layered 64x48 93 -> 72 us,
+            // 64^2 Poisson 134 -> 128 us); with fewer rows per wavefront it loses (32^2
+            // Poisson, 16 rows: 53 -> 64 us), and wide ILU(K) rows stay sync-free.
+            if (!h->identity && wl <= (double)SPCG_WCAP && h->n <= SPCG_RESIDENT_MAX_N && h->F.wL > 0 &&
+                (double)h->n / (double)h->F.wL >= 32.0)
+                strategy = SPCG_SPTRSV_RESIDENT;
         }
-        if (strategy < 1 || strategy > 3) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }
+        if (strategy < 1 || strategy > 4) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }
+        if (strategy == SPCG_SPTRSV_RESIDENT && h->n > SPCG_RESIDENT_MAX_N) {
+            delete h;
+            set_error("the resident executor holds every vector in one CTA's shared memory: n <= SPCG_RESIDENT_MAX_N");
+            return SPCG_ERR_INVALID_ARG;
+        }
         const int slots = sms * spcg_dev_ctas_per_sm();        // co-resident persistent CTAs
         int parts = opt.parts;
         if (parts <= 0) parts = h->n <= 16384 ? 1 : slots;
+        if (strategy == SPCG_SPTRSV_RESIDENT) parts = 1;
         parts = std::max(1, std::min<int>(parts, slots));
         if ((int64_t)parts > h->n) parts = (int)h->n;
         build_spmv_layout(h->A, h->lay.A);

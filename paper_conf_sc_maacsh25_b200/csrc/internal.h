@@ -80,7 +80,14 @@ struct TriLayout {
     std::vector<double> wval;
     std::vector<double> wdinv;     // [n] 1/u_ii per position (upper only)
     std::vector<int32_t> wgptr;    // [ngroups+1] position range of each level
+    // RESIDENT: one fixed 64-byte record per slice slot (slice s, lane l at s*32+l), so
+    // the kernel can stage a slice with four 16-byte cp.async per lane, addressed by the
+    // slot alone: {int32 (row+1) | level<<16, int32 len, double 1/u_ii, int32 col[4],
+    // double val[4]} (the vector fields 16-byte aligned).  Entries k >= 4 stay in src/val above (read through eoff).
+    std::vector<uint8_t> rrec;
 };
+constexpr int SPCG_RREC_BYTES = 64;
+constexpr int SPCG_RREC_PF = 4;
 
 struct SpmvLayout {                // SELL-32 of the original A, natural row order
     int32_t nslices = 0;

@@ -50,7 +50,8 @@ constexpr int BLOCK = SPCG_BLOCK;
 constexpr int NWARP = BLOCK / 32;
 constexpr long long SPIN_TIMEOUT_CYC = 8ll * 1000 * 1000 * 1000;            // ~4 s of SM cycles: abort, never hang
 
-enum { ST_LEVEL = SPCG_SPTRSV_LEVEL, ST_SYNCFREE = SPCG_SPTRSV_SYNCFREE, ST_CHUNKED = SPCG_SPTRSV_CHUNKED };
+enum { ST_LEVEL = SPCG_SPTRSV_LEVEL, ST_SYNCFREE = SPCG_SPTRSV_SYNCFREE, ST_CHUNKED = SPCG_SPTRSV_CHUNKED,
+       ST_RESIDENT = SPCG_SPTRSV_RESIDENT };
 enum { K_APPLY = 0, K_PRO = 1, K_ITER = 2 };
 enum { M_SOLVE = 0, M_SPMV = 1, M_LOWER = 2, M_UPPER = 3, M_PRECOND = 4 };
 
@@ -72,6 +73,7 @@ struct DevTri {
     const double* wval;
     const double* wdinv;
     const int32_t* wgptr;
+    const uint8_t* rrec;           // RESIDENT: 64-byte slot records (layout.cpp)
 };
 
 struct DevA {
@@ -626,12 +628,117 @@ __device__ void tri_syncfree_wide(const Params& P, const DevTri& T, int kind, co
     }
 }
 
+// RESIDENT executor's wavefront loop (one CTA; y/z and the fused operands in
+// shared memory).  Slice s belongs to warp s % NWARP, so consecutive wavefronts
+// (a single slice each on small 2-D grids) rotate over the warps.  A slice's
+// static data is one fixed 64-byte record per lane (row, level, length, the
+// first 4 dependency columns and values, 1/u_ii; layout.cpp), staged into a
+// per-warp double buffer in shared memory with cp.async two slices ahead: the
+// copies are asynchronous, so no warp stalls on a global load before a CTA
+// barrier (every warp must arrive at every barrier, so one stalled warp delays
+// the whole wavefront chain).  After a barrier only the staged-record read, the
+// shared-memory gathers, the FMA chain (k ascending, as the definition) and the
+// store remain.  The record's level tells a warp whether its next slice belongs
+// to the current wavefront; no level pointer is read.
+constexpr int RPF = SPCG_RREC_PF;
+constexpr int RES_STAGE_BYTES = NWARP * 2 * 32 * SPCG_RREC_BYTES;   // 32 KB
+__device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+                 "l"(gsrc)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+
+template <bool UPPER>
+__device__ void tri_resident(const Params& P, const DevTri& T, int kind, const double* in, double* out,
+                             const double* rdot, double alpha, double& acc_dot, double* stage) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t ns = T.nslices;
+    uint8_t* st = (uint8_t*)stage + (size_t)warp * 2 * 32 * SPCG_RREC_BYTES + lane * SPCG_RREC_BYTES;
+    auto issue = [&](int64_t sl, int b) {
+        if (sl < ns) {
+            const uint8_t* g = T.rrec + (size_t)(sl * 32 + lane) * SPCG_RREC_BYTES;
+            uint8_t* d = st + b * 32 * SPCG_RREC_BYTES;
+#pragma unroll
+            for (int q = 0; q < SPCG_RREC_BYTES / 16; ++q) cp_async16(d + 16 * q, g + 16 * q);
+        }
+        cp_async_commit();             // possibly empty: keeps the group count uniform
+    };
+    int64_t s = warp;
+    int buf = 0;
+    issue(s, 0);
+    issue(s + NWARP, 1);
+    for (int g = 0; g < T.ngroups; ++g) {
+        for (;;) {
+            if (s >= ns) break;
+            cp_async_wait1();          // slice s landed (s + NWARP may be in flight)
+            const uint8_t* R = st + buf * 32 * SPCG_RREC_BYTES;
+            const int w0 = *(const volatile int*)R;
+            if ((w0 >> 16) != g) break;  // warp-uniform: the level of my next slice
+            const int row = (w0 & 0xffff) - 1;
+            if (row >= 0) {
+                const int len = *(const int*)(R + 4);
+                const int4 cc = *(const int4*)(R + 16);
+                const double2 v01 = *(const double2*)(R + 32);
+                const double2 v23 = *(const double2*)(R + 48);
+                const int c[RPF] = {cc.x, cc.y, cc.z, cc.w};
+                const double v[RPF] = {v01.x, v01.y, v23.x, v23.y};
+                double acc;
+                if (!UPPER) {
+                    double ri;
+                    if (kind == K_ITER) {                       // Alg. 1 lines 11-12 fused
+                        ri = P.r[row] - alpha * P.w[row];
+                        P.r[row] = ri;
+                        P.x[row] = P.x[row] + alpha * P.p[row];
+                    } else {
+                        ri = in[row];
+                        if (kind == K_PRO) {
+                            if (in != P.r) P.r[row] = ri;
+                            if (!P.use_x0) P.x[row] = 0.0;
+                        }
+                    }
+                    acc_dot = fma(ri, ri, acc_dot);            // ||r||^2
+                    acc = ri;
+                } else {
+                    acc = in[row];
+                }
+                double d[RPF];
+#pragma unroll
+                for (int k = 0; k < RPF; ++k) d[k] = out[c[k]];
+#pragma unroll
+                for (int k = 0; k < RPF; ++k)
+                    if (k < len) acc = fma(-v[k], d[k], acc);
+                if (len > RPF) {
+                    const int64_t e0 = __ldg(T.eoff + s);
+                    for (int k = RPF; k < len; ++k)
+                        acc = fma(-__ldg(T.val + (e0 + k) * 32 + lane), out[-__ldg(T.src + (e0 + k) * 32 + lane) - 1], acc);
+                }
+                if (UPPER) {
+                    acc *= *(const double*)(R + 8);
+                    if (rdot) acc_dot = fma(rdot[row], acc, acc_dot);   // (r, z)
+                    if (kind == K_PRO) P.p[row] = acc;                   // p_0 = z_0
+                }
+                out[row] = acc;
+            }
+            __syncwarp();
+            issue(s + 2 * NWARP, buf);
+            buf ^= 1;
+            s += NWARP;
+        }
+        __syncthreads();
+    }
+    asm volatile("cp.async.wait_all;" ::: "memory");
+}
+
 template <int STRAT, bool UPPER>
 __device__ void tri_phase(const Params& P, const DevTri& T, int kind, const double* in, double* out,
                           const double* rdot, uint4* mb, unsigned ep, double alpha, double& acc_dot,
                           double* ring, unsigned& gen) {
     const int warp = threadIdx.x >> 5;
-    if (STRAT == ST_LEVEL && T.wide) {
+    if (STRAT == ST_RESIDENT) {
+        tri_resident<UPPER>(P, T, kind, in, out, rdot, alpha, acc_dot, ring);
+    } else if (STRAT == ST_LEVEL && T.wide) {
         tri_level_wide<UPPER>(P, T, kind, in, out, rdot, alpha, acc_dot, gen);
     } else if (STRAT == ST_SYNCFREE && T.wide) {
         tri_syncfree_wide<UPPER>(P, T, kind, in, out, rdot, mb, ep, alpha, acc_dot);
@@ -1552,8 +1659,7 @@ __device__ void tri_solve(const Params& P, int sec, int kind, const double* rin,
 }
 
 template <int STRAT>
-__global__ void __launch_bounds__(BLOCK, SPCG_CTAS_PER_SM) spcg_pcg_kernel(Params P) {
-    extern __shared__ __align__(128) double dyn[];
+__device__ __forceinline__ void pcg_body(const Params& P, double* dyn) {
     double* ring = dyn;
     unsigned gen = 0;
     if (threadIdx.x == 0) gen = ld_acquire_u32(&P.sc->bar_gen);
@@ -1657,6 +1763,45 @@ __global__ void __launch_bounds__(BLOCK, SPCG_CTAS_PER_SM) spcg_pcg_kernel(Param
     }
 }
 
+template <int STRAT>
+__global__ void __launch_bounds__(BLOCK, SPCG_CTAS_PER_SM) spcg_pcg_kernel(Params P) {
+    extern __shared__ __align__(128) double dyn[];
+    pcg_body<STRAT>(P, dyn);
+}
+
+// RESIDENT executor (small systems, n <= SPCG_RESIDENT_MAX_N): one CTA, every
+// vector of Algorithm 1 (x, r, w, p, y, z) held in shared memory for the whole
+// solve; the level-scheduled executor runs on them with CTA barriers between
+// wavefronts (grid_sync is a __syncthreads for a one-CTA grid), so a wavefront
+// handoff costs a CTA barrier (~15 ns) instead of a cross-CTA flag or a grid
+// barrier (0.3-1.2 us).  The factors and A stream from L1/L2.
+// b is read from global memory by the prologue; x is copied in (use_x0) and
+// out at the end.  The single-operator modes run on the caller's global buffers.
+__global__ void __launch_bounds__(BLOCK, 1) spcg_resident_kernel(Params P) {
+    extern __shared__ __align__(128) double dyn[];
+    if (P.mode != M_SOLVE) {
+        pcg_body<ST_RESIDENT>(P, dyn);
+        return;
+    }
+    const int64_t n = P.n;
+    double* gx = P.x;
+    Params Q = P;
+    Q.x = dyn;
+    Q.r = dyn + n;
+    Q.w = dyn + 2 * n;
+    Q.p = dyn + 3 * n;
+    Q.y = dyn + 4 * n;
+    Q.z = dyn + 5 * n;
+    if (P.use_x0)
+        for (int64_t i = threadIdx.x; i < n; i += BLOCK) Q.x[i] = gx[i];
+    __syncthreads();
+    pcg_body<ST_RESIDENT>(Q, dyn + 6 * n);
+    __syncthreads();
+    for (int64_t i = threadIdx.x; i < n; i += BLOCK) gx[i] = Q.x[i];
+}
+
+constexpr size_t resident_smem_bytes(int64_t n) { return (size_t)n * 6 * sizeof(double) + RES_STAGE_BYTES; }
+
 // ------------------------------------------------------------------ host side
 #define CK(call)                                                                              \
     do {                                                                                      \
@@ -1750,6 +1895,7 @@ static spcg_status_t upload_tri(spcg_device_t* d, const spcg::TriLayout& T, DevT
     if ((s = upload(d, T.wval, &D.wval))) return s;
     if ((s = upload(d, T.wdinv, &D.wdinv))) return s;
     if ((s = upload(d, T.wgptr, &D.wgptr))) return s;
+    if ((s = upload(d, T.rrec, &D.rrec))) return s;
     return SPCG_OK;
 }
 
@@ -1770,6 +1916,7 @@ static void* kernel_ptr() { return (void*)spcg_pcg_kernel<STRAT>; }
 
 static void* pick_kernel(int strategy) {
     switch (strategy) {
+        case ST_RESIDENT: return (void*)spcg_resident_kernel;
         case ST_LEVEL: return kernel_ptr<ST_LEVEL>();
         case ST_SYNCFREE: return kernel_ptr<ST_SYNCFREE>();
         default: return kernel_ptr<ST_CHUNKED>();
@@ -1822,10 +1969,14 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         spcg_dev_destroy(d);
         return SPCG_ERR_CUDA;
     }
-    d->smem = lay.strategy == ST_CHUNKED ? chunked_smem_bytes(lay.ring) : 0;
+    d->smem = lay.strategy == ST_CHUNKED    ? chunked_smem_bytes(lay.ring)
+              : lay.strategy == ST_RESIDENT ? resident_smem_bytes(n)
+                                            : 0;
     void* kfn = pick_kernel(d->strategy);
-    // one attribute value for every handle: the largest ring any layout builds
-    const int smem_max = lay.strategy == ST_CHUNKED ? (int)chunked_smem_bytes(SPCG_RING_MAX) : 0;
+    // one attribute value for every handle: the largest ring (or resident system) any layout builds
+    const int smem_max = lay.strategy == ST_CHUNKED    ? (int)chunked_smem_bytes(SPCG_RING_MAX)
+                         : lay.strategy == ST_RESIDENT ? (int)resident_smem_bytes(SPCG_RESIDENT_MAX_N)
+                                                       : 0;
     if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max) != cudaSuccess) {
         spcg::set_error("cannot reserve shared memory for the ring");
         spcg_dev_destroy(d);
@@ -1895,7 +2046,10 @@ static void report_abort(spcg_device_t* d, const Scal& sc) {
 static spcg_status_t launch(spcg_device_t* d, Params& P) {
     CK(cudaMemsetAsync(P.sc, 0, sizeof(Scal), d->stream));
     void* args[] = {&P};
-    CK(cudaLaunchCooperativeKernel(pick_kernel(d->strategy), dim3(d->parts), dim3(BLOCK), args, d->smem, d->stream));
+    if (d->strategy == ST_RESIDENT)   // one CTA: no co-residency requirement
+        CK(cudaLaunchKernel(pick_kernel(d->strategy), dim3(1), dim3(BLOCK), args, d->smem, d->stream));
+    else
+        CK(cudaLaunchCooperativeKernel(pick_kernel(d->strategy), dim3(d->parts), dim3(BLOCK), args, d->smem, d->stream));
     return SPCG_OK;
 }
 

@@ -189,6 +189,28 @@ static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev,
         }
     }
 
+    if (strategy == SPCG_SPTRSV_RESIDENT) {          // n <= SPCG_RESIDENT_MAX_N: 16-bit fields suffice
+        T.rrec.assign((size_t)ns * 32 * SPCG_RREC_BYTES, 0);
+        for (int32_t g = 0; g < T.ngroups; ++g)
+            for (int32_t s = T.gptr[g]; s < T.gptr[g + 1]; ++s)
+                for (int l = 0; l < 32; ++l) {
+                    uint8_t* R = T.rrec.data() + ((size_t)s * 32 + l) * SPCG_RREC_BYTES;
+                    const int32_t r = T.rows[(size_t)s * 32 + l];
+                    const int32_t w0 = (r + 1) | (g << 16);
+                    const int32_t len = r >= 0 ? (int32_t)(dep_end(r) - dep_begin(r)) : 0;
+                    memcpy(R, &w0, 4);
+                    memcpy(R + 4, &len, 4);
+                    for (int k = 0; k < SPCG_RREC_PF && k < len; ++k) {
+                        const int32_t j = M.col[dep_begin(r) + k];
+                        const double v = M.val[dep_begin(r) + k];
+                        memcpy(R + 16 + 4 * k, &j, 4);
+                        memcpy(R + 32 + 8 * k, &v, 8);
+                    }
+                    const double dv = (upper && r >= 0) ? 1.0 / M.val[M.rp[r]] : 0.0;
+                    memcpy(R + 8, &dv, 8);
+                }
+    }
+
     const size_t ne = (size_t)T.total_cols * 32;
     T.src.assign(ne, 0);
     T.val.assign(ne, 0.0);

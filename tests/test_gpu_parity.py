@@ -12,7 +12,13 @@ import paper_conf_sc_maacsh25_b200 as lib
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
-EXECUTORS = ["level", "syncfree", "chunked"]
+EXECUTORS = ["level", "syncfree", "chunked", "resident"]
+
+
+def _fits(ex, A):
+    """The resident executor takes n <= RESIDENT_MAX_N (one CTA's shared memory)."""
+    if ex == "resident" and A.n > lib.RESIDENT_MAX_N:
+        pytest.skip("resident executor: n > RESIDENT_MAX_N")
 
 
 def _dev(a):
@@ -33,6 +39,7 @@ SMALL = [("poisson2d", (37, 29), 0), ("poisson3d", (13, 11, 9), 0), ("fem_q1", (
 @pytest.mark.parametrize("parts", [1, 7, 0])
 def test_operators_match_oracle(fam, params, K, ex, parts):
     A = gen.make(fam, *params)
+    _fits(ex, A)
     h = lib.SPCG(A, mode="alg2", K=K, sptrsv=ex, parts=parts)
     L, U, _ = oracle.setup(A, mode="alg2", K=K)
     rng = np.random.default_rng(5)
@@ -68,6 +75,7 @@ def test_operators_match_oracle(fam, params, K, ex, parts):
 @pytest.mark.parametrize("ex", EXECUTORS)
 def test_pcg_matches_oracle(fam, params, K, mode, ex):
     A = gen.make(fam, *params)
+    _fits(ex, A)
     b, xt = gen.rhs(A)
     h = lib.SPCG(A, mode=mode, K=K, sptrsv=ex)
     L, U, _ = oracle.setup(A, mode=mode, K=K)
@@ -104,7 +112,7 @@ def test_identity_preconditioner_is_cg():
 
 @pytest.mark.parametrize("ex", EXECUTORS)
 def test_deterministic_bitwise(ex):
-    A = gen.make("aniso_layered", 300, 211, 4)
+    A = gen.make("aniso_layered", 300, 211, 4) if ex != "resident" else gen.make("aniso_layered", 64, 60, 4)
     b, _ = gen.rhs(A)
     h = lib.SPCG(A, sptrsv=ex)
     x1, i1 = h.solve(_dev(b), eps=1e-8, kmax=5000)
@@ -197,7 +205,7 @@ def test_degenerate_cases(ex):
     x, info = h.solve(_dev(b), eps=1e-8, kmax=0)
     assert info["iterations"] == 0 and info["status"] == lib.NOT_CONVERGED and not torch.any(x != 0)
     h.close()
-    for d in (np.array([[3.0]]), np.diag(np.linspace(1.0, 7.0, 5000))):
+    for d in (np.array([[3.0]]), np.diag(np.linspace(1.0, 7.0, 5000 if ex != "resident" else 4096))):
         Ad = gen.from_dense(d) if d.shape[0] == 1 else gen.CSR(d.shape[0], np.arange(d.shape[0] + 1, dtype=np.int64),
                                                                np.arange(d.shape[0], dtype=np.int32), np.diag(d).copy())
         bd = np.linspace(-1.0, 1.0, Ad.n) if Ad.n > 1 else np.array([1.5])
@@ -207,3 +215,23 @@ def test_degenerate_cases(ex):
         assert info["iterations"] == 1 and info["status"] == 0
         assert np.allclose(xd.cpu().numpy(), bd / np.diag(d), rtol=1e-15, atol=0)
         hd.close()
+
+
+def test_resident_limits_and_initial_guess():
+    """RESIDENT executor: the largest system it takes (n = RESIDENT_MAX_N, 64x64
+    Poisson) matches the oracle in forced-k mode from a user x0 (x copied in and out
+    of shared memory); one row more is rejected with INVALID_ARG at setup."""
+    A = gen.make("poisson2d", 64, 64)
+    assert A.n == lib.RESIDENT_MAX_N
+    b, xt = gen.rhs(A)
+    h = lib.SPCG(A, sptrsv="resident")
+    assert h.info["sptrsv_name"] == "resident" and h.info["parts"] == 1
+    L, U, _ = oracle.setup(A, mode="alg2", K=0)
+    x0 = 0.25 * xt
+    ro = oracle.pcg(A, L, U, b, 0.0, 9, x0=x0)
+    xg = _dev(x0)
+    h.solve(_dev(b), xg, eps=0.0, kmax=9, use_x0=True)
+    assert np.linalg.norm(xg.cpu().numpy() - ro["x"]) <= 1e-10 * np.linalg.norm(ro["x"])
+    h.close()
+    with pytest.raises(lib.SpcgError):
+        lib.SPCG(gen.make("poisson2d", 65, 64), sptrsv="resident")

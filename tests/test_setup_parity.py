@@ -169,3 +169,16 @@ def test_setup_info_bytes_formula():
     assert i["algo_bytes_per_iter"] == expect
     assert i["levels_L"] == 28 and i["levels_U"] == 28
     h.close()
+
+
+def test_resident_executor_host_checks():
+    """RESIDENT (one CTA, vectors in shared memory) is accepted up to
+    RESIDENT_MAX_N rows, runs as one part, and is refused above (INVALID_ARG at
+    setup, before any device work)."""
+    A = gen.make("poisson2d", 64, 64)
+    h = lib.SPCG(A, mode="none", sptrsv="resident", parts=9, device=-1)
+    assert h.info["sptrsv_name"] == "resident" and h.info["parts"] == 1
+    assert h.info["levels_L"] == 127                 # nx + ny - 1 (P2)
+    h.close()
+    with pytest.raises(lib.SpcgError):
+        lib.SPCG(gen.make("poisson2d", 65, 64), sptrsv="resident", device=-1)

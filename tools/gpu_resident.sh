@@ -1,0 +1,6 @@
+# resident executor: GPU parity + small-system executor comparison + C1 bench
+O=gpurun_out/r01e_res; mkdir -p $O
+python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1; echo "build rc=$?"
+timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -m gpu > $O/pytest_parity.log 2>&1; echo "pytest rc=$?"; tail -3 $O/pytest_parity.log
+timeout 600 python tools/res_cmp.py > $O/res_cmp.jsonl 2> $O/res_cmp.err; echo "cmp rc=$?"; cat $O/res_cmp.jsonl
+timeout 300 python bench.py --workload C1 --sptrsv resident > $O/bench_c1_resident.json 2> $O/bench_c1.err; echo "c1 rc=$?"
