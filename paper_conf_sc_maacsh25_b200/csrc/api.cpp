@@ -158,13 +158,12 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         if (strategy == SPCG_SPTRSV_AUTO) {
             const double wl = h->n > 0 ? (double)h->F.L.nnz() / (double)h->n : 0.0;
             strategy = (h->identity || wl <= (double)SPCG_WCAP) ? SPCG_SPTRSV_CHUNKED : SPCG_SPTRSV_SYNCFREE;
-            // Small systems with >= 32 rows per wavefront on average: the one-CTA resident
-            // executor (vectors in shared memory, CTA barriers) beats the chunked pipeline
-            // (measured per iteration: 16^3 Poisson 129 -> 63 us, layered 64x48 93 -> 72 us,
-            // 64^2 Poisson 134 -> 128 us); with fewer rows per wavefront it loses (32^2
-            // Poisson, 16 rows: 53 -> 64 us), and wide ILU(K) rows stay sync-free.
-            if (!h->identity && wl <= (double)SPCG_WCAP && h->n <= SPCG_RESIDENT_MAX_N && h->F.wL > 0 &&
-                (double)h->n / (double)h->F.wL >= 32.0)
+            // Small systems: the one-CTA resident executor (vectors in shared memory, CTA
+            // barriers) beats the chunked pipeline on every narrow case measured (per
+            // iteration: 32^2 Poisson 53 -> 46 us, 64^2 Poisson 133 -> 90, 16^3 Poisson
+            // 129 -> 49, layered 64x48 93 -> 54); wide ILU(K) rows stay sync-free
+            // (DESIGN.md §5.3).
+            if (!h->identity && wl <= (double)SPCG_WCAP && h->n <= SPCG_RESIDENT_MAX_N)
                 strategy = SPCG_SPTRSV_RESIDENT;
         }
         if (strategy < 1 || strategy > 4) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }

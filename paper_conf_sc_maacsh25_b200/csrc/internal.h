@@ -82,12 +82,14 @@ struct TriLayout {
     std::vector<int32_t> wgptr;    // [ngroups+1] position range of each level
     // RESIDENT: one fixed 64-byte record per slice slot (slice s, lane l at s*32+l), so
     // the kernel can stage a slice with four 16-byte cp.async per lane, addressed by the
-    // slot alone: {int32 (row+1) | level<<16, int32 len, double 1/u_ii, int32 col[4],
-    // double val[4]} (the vector fields 16-byte aligned).  Entries k >= 4 stay in src/val above (read through eoff).
+    // slot alone: {int32 (row+1) | level<<16, int32 len | next<<16, double 1/u_ii,
+    // int32 col[4], double val[4]} (the vector fields 16-byte aligned); next = level of
+    // slice s + SPCG_RES_WARPS (the same warp's next slice; 0xffff: none).  Entries k >= 4 stay in src/val above (read through eoff).
     std::vector<uint8_t> rrec;
 };
 constexpr int SPCG_RREC_BYTES = 64;
 constexpr int SPCG_RREC_PF = 4;
+constexpr int SPCG_RES_WARPS = 8;      // warps of the resident CTA (slice s -> warp s % 8)
 
 struct SpmvLayout {                // SELL-32 of the original A, natural row order
     int32_t nslices = 0;

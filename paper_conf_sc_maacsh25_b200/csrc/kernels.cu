@@ -650,6 +650,7 @@ __device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc) {
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 
+static_assert(NWARP >= SPCG_RES_WARPS, "the resident executor deals slices over 8 warps (layout.cpp records)");
 template <bool UPPER>
 __device__ void tri_resident(const Params& P, const DevTri& T, int kind, const double* in, double* out,
                              const double* rdot, double alpha, double& acc_dot, double* stage) {
@@ -667,18 +668,27 @@ __device__ void tri_resident(const Params& P, const DevTri& T, int kind, const d
     };
     int64_t s = warp;
     int buf = 0;
+    const bool owner = warp < SPCG_RES_WARPS;
+    if (!owner) s = ns;
     issue(s, 0);
-    issue(s + NWARP, 1);
+    issue(s + SPCG_RES_WARPS, 1);
+    // level of my next slice: read once here, then carried in each record (the
+    // owner of a wavefront goes from its store straight to the barrier)
+    int gnext = 0xffff;
+    if (s < ns) {
+        cp_async_wait1();
+        gnext = (*(const volatile int*)st) >> 16;
+    }
     for (int g = 0; g < T.ngroups; ++g) {
-        for (;;) {
-            if (s >= ns) break;
-            cp_async_wait1();          // slice s landed (s + NWARP may be in flight)
+        while (gnext == g) {           // warp-uniform
+            cp_async_wait1();          // slice s landed (s + 8 may be in flight)
             const uint8_t* R = st + buf * 32 * SPCG_RREC_BYTES;
-            const int w0 = *(const volatile int*)R;
-            if ((w0 >> 16) != g) break;  // warp-uniform: the level of my next slice
+            const int w0 = *(const int*)R;
+            const int w1 = *(const int*)(R + 4);
+            gnext = w1 >> 16;
             const int row = (w0 & 0xffff) - 1;
             if (row >= 0) {
-                const int len = *(const int*)(R + 4);
+                const int len = w1 & 0xffff;
                 const int4 cc = *(const int4*)(R + 16);
                 const double2 v01 = *(const double2*)(R + 32);
                 const double2 v23 = *(const double2*)(R + 48);
@@ -721,10 +731,9 @@ __device__ void tri_resident(const Params& P, const DevTri& T, int kind, const d
                 }
                 out[row] = acc;
             }
-            __syncwarp();
-            issue(s + 2 * NWARP, buf);
+            issue(s + 2 * SPCG_RES_WARPS, buf);
             buf ^= 1;
-            s += NWARP;
+            s += SPCG_RES_WARPS;
         }
         __syncthreads();
     }

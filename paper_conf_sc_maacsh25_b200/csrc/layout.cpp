@@ -191,6 +191,9 @@ static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev,
 
     if (strategy == SPCG_SPTRSV_RESIDENT) {          // n <= SPCG_RESIDENT_MAX_N: 16-bit fields suffice
         T.rrec.assign((size_t)ns * 32 * SPCG_RREC_BYTES, 0);
+        std::vector<int32_t> lev_of(ns, 0);
+        for (int32_t g = 0; g < T.ngroups; ++g)
+            for (int32_t s = T.gptr[g]; s < T.gptr[g + 1]; ++s) lev_of[s] = g;
         for (int32_t g = 0; g < T.ngroups; ++g)
             for (int32_t s = T.gptr[g]; s < T.gptr[g + 1]; ++s)
                 for (int l = 0; l < 32; ++l) {
@@ -198,8 +201,10 @@ static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev,
                     const int32_t r = T.rows[(size_t)s * 32 + l];
                     const int32_t w0 = (r + 1) | (g << 16);
                     const int32_t len = r >= 0 ? (int32_t)(dep_end(r) - dep_begin(r)) : 0;
+                    const int32_t nxt = s + SPCG_RES_WARPS < ns ? lev_of[s + SPCG_RES_WARPS] : 0xffff;
+                    const int32_t w1 = len | (nxt << 16);
                     memcpy(R, &w0, 4);
-                    memcpy(R + 4, &len, 4);
+                    memcpy(R + 4, &w1, 4);
                     for (int k = 0; k < SPCG_RREC_PF && k < len; ++k) {
                         const int32_t j = M.col[dep_begin(r) + k];
                         const double v = M.val[dep_begin(r) + k];
