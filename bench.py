@@ -336,7 +336,9 @@ def main():
                         "per_iter_speedup": (p_ms / max(p["k"], 1)) / (s_ms / max(s["k"], 1))},
         "paper_context": PAPER_CONTEXT,
         "roofline": {"bound": "hbm", "achieved": s_gbs, "peak": peak, "unit": "GB/s", "frac": s_gbs / peak,
-                     "traffic": traffic, "kernel": "spcg_pcg_kernel (persistent, whole Alg. 1)",
+                     "traffic": traffic,
+                     "kernel": ("spcg_resident_kernel (one CTA, whole Alg. 1)" if si["sptrsv_name"] == "resident"
+                                else "spcg_pcg_kernel (persistent, whole Alg. 1)"),
                      "peak_source": peak_src,
                      "achieved_def": "B_iter (DESIGN.md §4) x iterations / CUDA-event time of the launch",
                      "l2_hit_pct": l2_hit,
