@@ -111,7 +111,8 @@ def setup_rank(systems, device: int, mode: str = "alg2", lanes: int = 1, sms: in
         extra = dict(kw)
         if streams is not None:
             extra["stream"] = streams[lane_of[s.index]]
-            extra["parts"] = 1 if A.n <= 16384 else max(1, sms // lanes)
+            # one CTA for small narrow systems; wide ILU(K) rows (sync-free) take the lane's CTAs
+            extra["parts"] = 1 if (A.n <= 16384 and s.K == 0) else max(1, sms // lanes)
         h = SPCG(A, mode=mode, K=s.K, device=device, **extra)
         h.lane = lane_of.get(s.index, 0)
         handles.append((s, A, b, h, time.perf_counter() - t0))

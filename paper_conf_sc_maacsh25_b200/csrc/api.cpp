@@ -174,7 +174,10 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         }
         const int slots = sms * spcg_dev_ctas_per_sm();        // co-resident persistent CTAs
         int parts = opt.parts;
-        if (parts <= 0) parts = h->n <= 16384 ? 1 : slots;
+        // small systems: one CTA, except sync-free (wide ILU(K) rows), whose rows of a
+        // wavefront spread over every warp of the grid (FEM 20^3 ILU(2), per iteration:
+        // 1 CTA 2.38 ms, 37 CTAs 0.81 ms; profiles/r01_final/fem_parts.jsonl)
+        if (parts <= 0) parts = (h->n <= 16384 && strategy != SPCG_SPTRSV_SYNCFREE) ? 1 : slots;
         if (strategy == SPCG_SPTRSV_RESIDENT) parts = 1;
         parts = std::max(1, std::min<int>(parts, slots));
         if ((int64_t)parts > h->n) parts = (int)h->n;
