@@ -111,8 +111,13 @@ def setup_rank(systems, device: int, mode: str = "alg2", lanes: int = 1, sms: in
         extra = dict(kw)
         if streams is not None:
             extra["stream"] = streams[lane_of[s.index]]
-            # one CTA for small narrow systems; wide ILU(K) rows (sync-free) take the lane's CTAs
-            extra["parts"] = 1 if (A.n <= 16384 and s.K == 0) else max(1, sms // lanes)
+            # narrow systems: one CTA up to 4096 rows (resident), 16 up to 16384 (chunked,
+            # DESIGN.md §5); larger ones and wide ILU(K) rows (sync-free) take the lane's CTAs
+            lane_ctas = max(1, sms // lanes)
+            if A.n <= 16384 and s.K == 0:
+                extra["parts"] = 1 if A.n <= 4096 else min(16, lane_ctas)
+            else:
+                extra["parts"] = lane_ctas
         h = SPCG(A, mode=mode, K=s.K, device=device, **extra)
         h.lane = lane_of.get(s.index, 0)
         handles.append((s, A, b, h, time.perf_counter() - t0))

@@ -177,7 +177,15 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         // small systems: one CTA, except sync-free (wide ILU(K) rows), whose rows of a
         // wavefront spread over every warp of the grid (FEM 20^3 ILU(2), per iteration:
         // 1 CTA 2.38 ms, 37 CTAs 0.81 ms; profiles/r01_final/fem_parts.jsonl)
-        if (parts <= 0) parts = (h->n <= 16384 && strategy != SPCG_SPTRSV_SYNCFREE) ? 1 : slots;
+        // Mid-size narrow systems (4096 < n <= 16384) take 16 CTAs: one CTA walks every
+        // wavefront alone, 16 let the inspector split the chains (components / strided /
+        // tiles); per iteration, layered 90x91 231 -> 84 us, 25^3 Poisson 487 -> 169 us,
+        // 128^2 Poisson 449 -> 298 us (profiles/r01_final/mid_parts.jsonl; 16 has the
+        // smallest sum over the four cases of 1..37).
+        if (parts <= 0) {
+            if (strategy == SPCG_SPTRSV_SYNCFREE || h->n > 16384) parts = slots;
+            else parts = (h->n <= 4096 || h->identity) ? 1 : std::min(16, slots);
+        }
         if (strategy == SPCG_SPTRSV_RESIDENT) parts = 1;
         parts = std::max(1, std::min<int>(parts, slots));
         if ((int64_t)parts > h->n) parts = (int)h->n;
