@@ -438,7 +438,12 @@ def run_batch(args, ws, rank, local):
         r = batch.solve_rank(hs)
         return r, sum(x.iter_phase_ms for x in r)
 
+    last = None
     for _ in range(max(1, args.warmup)):
+        last = step()
+    if args.lanes > 1 and args.sched == "static":
+        # static lanes re-planned by LPT over the warm-up step's measured per-system times
+        batch.replan_lanes(hs, {x.index: x.iter_phase_ms for x in last[0]}, args.lanes)
         step()
     t_dev = []
     clk = Clocks(local)
@@ -481,7 +486,9 @@ def run_batch(args, ws, rank, local):
                 "dtype": "f64", "data": "synthetic",
                 "config": {"workload": WORKLOADS["C5"], "systems": len(systems), "eps": EPS, "lanes": args.lanes,
                            "makespan": (f"device events fork/join around the rank's solves ({args.sched} lanes: "
-                                        f"{args.lanes} streams x {sms // args.lanes} CTAs)" if args.lanes > 1 else
+                                        f"{args.lanes} streams x {sms // args.lanes} CTAs"
+                                        + ("; lanes re-planned by LPT over the warm-up step's measured per-system times)"
+                                           if args.sched == "static" else ")") if args.lanes > 1 else
                                         "sum of the rank's device-timed solves (back to back)") +
                                        "; max over ranks",
                            "l2": "no flush: 64 different systems run back to back (working set >> L2)"},

@@ -185,6 +185,26 @@ def solve_rank_dynamic(handles, lanes: int, eps: float = 1e-8, kmax: int = 20000
     return sorted(out, key=lambda r: r.index), float(t0.elapsed_time(t1))
 
 
+def replan_lanes(handles, measured_ms, lanes: int):
+    """LPT of this rank's systems over its lanes by MEASURED solve times (SURVEY
+    §8(e): the cost estimates refined by the measured per-system times, here those
+    of a warm-up step).  Handles are rebound with spcg_set_stream (device-side
+    ordering, the host does not block).  Returns the per-lane load (ms)."""
+    by_lane = {}
+    for item in handles:
+        by_lane.setdefault(item[3].lane, item[3].stream)
+    streams = [by_lane[k] for k in sorted(by_lane)]
+    load = [0.0] * len(streams)
+    for it in sorted(handles, key=lambda it: (-measured_ms[it[0].index], it[0].index)):
+        k = min(range(len(streams)), key=lambda j: (load[j], j))
+        load[k] += measured_ms[it[0].index]
+        h = it[3]
+        if h.stream is not streams[k]:
+            h.set_stream(streams[k])
+        h.lane = k
+    return load
+
+
 def solve_rank_concurrent(handles, eps: float = 1e-8, kmax: int = 20000):
     """All of this rank's systems in flight at once, one stream per lane
     (spcg_solve_async / spcg_solve_wait).  Returns (results, device makespan ms):

@@ -81,3 +81,29 @@ def test_gather_two_ranks_gloo():
         import paper_conf_sc_maacsh25_b200 as lib
         h = lib.SPCG(A, K=s.K, device=-1)
         assert o[1] == A.n and o[2] == h.info["levels_L"] and o[3] == h.info["chosen_pct"]
+
+
+def test_replan_lanes_lpt_by_measured_times():
+    """C5 re-planning: systems go, longest measured time first, to the
+    least-loaded lane; handles whose lane changes are rebound with set_stream."""
+    from types import SimpleNamespace
+    from paper_conf_sc_maacsh25_b200 import batch
+
+    class H:
+        def __init__(self, lane, stream):
+            self.lane, self.stream, self.rebound = lane, stream, 0
+
+        def set_stream(self, st):
+            self.stream, self.rebound = st, self.rebound + 1
+
+    streams = [object(), object()]
+    ms = {0: 10.0, 1: 9.0, 2: 6.0, 3: 5.0, 4: 1.0}
+    handles = [(SimpleNamespace(index=i), None, None, H(0, streams[0]), 0.0) for i in ms]   # all on lane 0
+    handles[1][3].lane, handles[1][3].stream = 1, streams[1]
+    load = batch.replan_lanes(handles, ms, 2)
+    assert sorted(load) == [15.0, 16.0]                       # LPT: {10, 5, 1} / {9, 6}
+    lanes = {it[0].index: it[3].lane for it in handles}
+    assert lanes[0] == 0 and lanes[1] == 1 and lanes[2] == 1 and lanes[3] == 0 and lanes[4] == 0
+    for it in handles:
+        assert it[3].stream is streams[it[3].lane]
+    assert handles[2][3].rebound == 1 and handles[0][3].rebound == 0
