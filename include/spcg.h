@@ -142,6 +142,10 @@ typedef struct {
     double total_ms;            /* including host<->device copies when SPCG_HOST_PTRS */
 } spcg_solve_info_t;
 
+/* Largest kmax a solve accepts (SPCG_ERR_INVALID_ARG above it): the device's
+ * per-solve ready-flag epochs are 32-bit and advance by kmax + 3 per solve. */
+#define SPCG_KMAX_LIMIT 1000000000LL
+
 /* spcg_solve flags */
 #define SPCG_USE_X0 0x1u        /* x holds the initial guess (default x0 = 0) */
 #define SPCG_HOST_PTRS 0x2u     /* b and x are HOST pointers: copies happen inside the call */

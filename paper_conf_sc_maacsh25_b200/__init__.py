@@ -246,12 +246,26 @@ class SPCG:
         return L, U
 
     # ------------------------------------------------------------ solve
+    def _order_after_current(self, *tensors):
+        """The handle's stream waits (on the device) for the caller's current stream, where
+        b / x were produced; tensors used asynchronously are recorded on the handle's stream
+        so the caching allocator does not recycle them early."""
+        torch = _torch()
+        cur = torch.cuda.current_stream(self.device)
+        if cur.cuda_stream != self.stream.cuda_stream:
+            ev = torch.cuda.Event()
+            ev.record(cur)
+            self.stream.wait_event(ev)
+            for t in tensors:
+                t.record_stream(self.stream)
+
     def solve(self, b, x=None, eps=1e-8, kmax=10000, use_x0=False):
         """b, x: float64 CUDA tensors of length n on this handle's device (x allocated if None)."""
         torch = _torch()
         assert b.dtype == torch.float64 and b.is_cuda and b.is_contiguous() and b.numel() == self.n
         if x is None:
             x = torch.empty_like(b)
+        self._order_after_current(b, x)
         info = SolveInfo()
         flags = USE_X0 if use_x0 else 0
         st = load().spcg_solve(self._h, b.data_ptr(), x.data_ptr(), float(eps), int(kmax), flags, ctypes.byref(info))
@@ -260,6 +274,7 @@ class SPCG:
 
     def solve_async(self, b, x, eps=1e-8, kmax=10000):
         """spcg_solve_async: enqueue on the handle's stream (b, x device tensors kept alive by the caller)."""
+        self._order_after_current(b, x)
         _check(load().spcg_solve_async(self._h, b.data_ptr(), x.data_ptr(), float(eps), int(kmax), 0),
                "spcg_solve_async")
 

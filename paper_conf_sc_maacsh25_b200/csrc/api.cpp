@@ -266,6 +266,7 @@ spcg_status_t spcg_get_setup_info(spcg_handle_t h, spcg_setup_info_t* info) {
 spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps, int64_t kmax,
                          uint32_t flags, spcg_solve_info_t* info) {
     if (!h || !b || !x || kmax < 0 || !(eps >= 0.0)) { set_error("bad solve arguments"); return SPCG_ERR_INVALID_ARG; }
+    if (kmax > SPCG_KMAX_LIMIT) { set_error("kmax > SPCG_KMAX_LIMIT"); return SPCG_ERR_INVALID_ARG; }
     if (!h->dev) { set_error("host-only handle"); return SPCG_ERR_NO_DEVICE; }
     spcg_solve_info_t tmp{};
     spcg_solve_info_t* I = info ? info : &tmp;
@@ -279,10 +280,19 @@ spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps
             st = spcg_dev_copy(h->dev, &db, nullptr, 0, -1);    // the handle's staging buffer (b | x)
             if (st != SPCG_OK) return st;
             double* dx = db + h->n;
-            spcg_dev_copy(h->dev, db, b, (size_t)h->n * 8, 1);
-            if (flags & SPCG_USE_X0) spcg_dev_copy(h->dev, dx, x, (size_t)h->n * 8, 1);
+            st = spcg_dev_copy(h->dev, db, b, (size_t)h->n * 8, 1);
+            if (st != SPCG_OK) return st;
+            if (flags & SPCG_USE_X0) {
+                st = spcg_dev_copy(h->dev, dx, x, (size_t)h->n * 8, 1);
+                if (st != SPCG_OK) return st;
+            }
             st = spcg_dev_solve(h->dev, db, dx, eps, kmax, (flags & SPCG_USE_X0) != 0, I, &h->rhist);
-            spcg_dev_copy(h->dev, x, dx, (size_t)h->n * 8, 2);
+            // x is written back only when the kernel ran (it then holds x_k, Alg. 1 line 17);
+            // on a launch/argument error the caller's x stays untouched
+            if (st == SPCG_OK || st == SPCG_NOT_CONVERGED || st == SPCG_ERR_BREAKDOWN) {
+                spcg_status_t cs = spcg_dev_copy(h->dev, x, dx, (size_t)h->n * 8, 2);
+                if (cs != SPCG_OK) return cs;
+            }
         } else {
             st = spcg_dev_solve(h->dev, b, x, eps, kmax, (flags & SPCG_USE_X0) != 0, I, &h->rhist);
         }
@@ -298,6 +308,7 @@ spcg_status_t spcg_solve_async(spcg_handle_t h, const double* b, double* x, doub
                                uint32_t flags) {
     if (!h || !b || !x || kmax < 0 || !(eps >= 0.0)) { set_error("bad solve arguments"); return SPCG_ERR_INVALID_ARG; }
     if (flags & SPCG_HOST_PTRS) { set_error("spcg_solve_async takes device pointers only"); return SPCG_ERR_INVALID_ARG; }
+    if (kmax > SPCG_KMAX_LIMIT) { set_error("kmax > SPCG_KMAX_LIMIT"); return SPCG_ERR_INVALID_ARG; }
     if (!h->dev) { set_error("host-only handle"); return SPCG_ERR_NO_DEVICE; }
     try {
         return spcg_dev_solve_begin(h->dev, b, x, eps, kmax, (flags & SPCG_USE_X0) != 0);

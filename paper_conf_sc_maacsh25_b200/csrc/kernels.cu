@@ -887,6 +887,13 @@ __device__ __forceinline__ bool warp_ok(bool ok) { return __all_sync(0xffffffffu
 // in order).  No fence on the solver's critical path.
 __device__ __forceinline__ void fence_acq_rel_cta() { asm volatile("fence.acq_rel.cta;" ::: "memory"); }
 __device__ __forceinline__ double lds_volatile(const double* p) { return *(const volatile double*)p; }
+// the solver's read of the poller's mask: an acquire load (CTA scope) pairs with the
+// poller's fence.acq_rel + atomicOr, so the value load after it sees the value store
+__device__ __forceinline__ unsigned lds_acquire_u32(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+    return v;
+}
 // After an abort the ring may hold stale chunks: roles must stop parsing them.
 // Warp-collective code must take this decision warp-uniformly (a per-lane read
 // of a racy flag lets lanes disagree; a divergent break then deadlocks the
@@ -1127,7 +1134,7 @@ __device__ __noinline__ double2 slow_record(const uint8_t* p, int fl, int wd, in
     if (fl & REC_FIRST) {
         double e = 0.0;
         if (row >= 0 && ne > 0) {
-            const unsigned m = *(volatile unsigned*)(side_rec + 96);
+            const unsigned m = lds_acquire_u32((const unsigned*)(side_rec + 96));
             if (m & (1u << lane)) e = lds_volatile(side_rec + 64 + lane);
             else e = ext_wait(R, lane, ne, mb, ep, sc);
         }
@@ -1186,7 +1193,7 @@ __device__ __forceinline__ void solve_record(const SolveCtx& C, const Prep& X, i
     } else if ((X.fl & (REC_FIRST | REC_WIDE)) == REC_FIRST) {
         // cross-CTA terms: normally pre-resolved by the poller into the side slot
         const int ne = meta_ne(X.meta);
-        const unsigned m = *(volatile unsigned*)side_mask(*C.S, slot, X.r);
+        const unsigned m = lds_acquire_u32(side_mask(*C.S, slot, X.r));
         const bool have = ne == 0 || (m >> lane) & 1u;
         const bool all_have = __all_sync(0xffffffffu, have);
         if (SPCG_DEBUG_COUNTS && g_dbg_counts && lane == 0) atomicAdd(g_dbg_counts + (all_have ? 1 : 2), 1ull);
@@ -2052,6 +2059,18 @@ static void report_abort(spcg_device_t* d, const Scal& sc) {
     spcg::set_error(buf);
 }
 
+// Ready-flag epochs are 32-bit and advance by kmax + 3 per solve (kmax <= SPCG_KMAX_LIMIT).
+// Before they could wrap, the flag arrays are re-initialised on the stream (0xFF..: the
+// epoch 0xFFFFFFFF is never issued) and numbering restarts at 1, so a stale flag can
+// never carry a current epoch.
+static spcg_status_t reserve_epochs(spcg_device_t* d, unsigned long long need) {
+    if ((unsigned long long)d->epoch + need < 0xFFFFFF00ull) return SPCG_OK;
+    CK(cudaMemsetAsync(d->P.mbL, 0xFF, (size_t)d->P.n * 16, d->stream));
+    CK(cudaMemsetAsync(d->P.mbU, 0xFF, (size_t)d->P.n * 16, d->stream));
+    d->epoch = 1;
+    return SPCG_OK;
+}
+
 static spcg_status_t launch(spcg_device_t* d, Params& P) {
     CK(cudaMemsetAsync(P.sc, 0, sizeof(Scal), d->stream));
     void* args[] = {&P};
@@ -2076,6 +2095,10 @@ spcg_status_t spcg_dev_solve_begin(spcg_device_t* d, const double* b, double* x,
     P.eps = eps;
     P.kmax = kmax;
     P.use_x0 = use_x0 ? 1 : 0;
+    {
+        spcg_status_t es = reserve_epochs(d, (unsigned long long)kmax + 3ull);
+        if (es != SPCG_OK) return es;
+    }
     P.epoch = d->epoch;
     d->epoch += (unsigned)(kmax + 3);
     long long cap = std::min<long long>(kmax + 1, 1 << 20);
@@ -2165,6 +2188,10 @@ spcg_status_t spcg_dev_apply(spcg_device_t* d, int op, const double* in, double*
     P.in = in;
     P.out = out;
     P.aux = aux;
+    {
+        spcg_status_t es = reserve_epochs(d, 1ull);
+        if (es != SPCG_OK) return es;
+    }
     P.epoch = d->epoch;
     d->epoch += 1;
     P.rhist = nullptr;
