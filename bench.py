@@ -4,15 +4,19 @@
 Metric: "SPCG iter-phase ms to eps=1e-8 + HBM GB/s per iter vs unsparsified PCG".
 A *step* is one full pass of the hot path: one solve of Algorithm 1 (prologue +
 iterations to ||r|| < 1e-8) on the workload, inputs resident in HBM.  The
-default workload is BASELINE.json configs[1] (C2: 3D 7-point Poisson 64^3,
-ILU(0), SPCG = Algorithm 2 vs PCG = no sparsification).
+default workload at N = 1 is the largest single-GPU config of BASELINE.json,
+C4 (2-D layered anisotropic diffusion 4096^2, n = 16.8 M, ILU(0); SPCG =
+Algorithm 2 vs PCG = no sparsification, plus the fixed-t sweep t in {1,5,10}),
+where the working set (4.2 GB per iteration) is far beyond L2 and the HBM
+roofline applies.  C1-C3 stay selectable (--workload).  At N > 1 the default is
+the C5 batch (64 independent systems, LPT over the ranks: strong scaling).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--sptrsv auto]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C4] [--sptrsv auto]
   python bench.py --impl reference ...      # the oracle (plain fp64 C, host cores)
 
-N > 1 (torchrun): every rank solves its own replica of the workload (a single
-system does not shard: DESIGN.md §7), no collective on the data path; times are
-max over ranks.
+N > 1 with C1-C4 (torchrun): every rank solves its own replica (a single system
+does not shard: DESIGN.md §7), no collective on the data path; times are max
+over ranks.
 """
 from __future__ import annotations
 
@@ -130,41 +134,74 @@ def _cpu_info():
     return model
 
 
-def run_oracle(name: str, A, b, steps: int, warmup: int, budget_s: float = 20.0, k_hint=None):
-    """The oracle as it stands (single thread, plain C), timed on the host.
+def _kref():
+    """The oracle's own iteration counts to eps (oracle/kref.json, written by
+    tools/oracle_kref.py from one full single-thread oracle solve per config/mode)."""
+    p = os.path.join(ROOT, "oracle", "kref.json")
+    return json.load(open(p)) if os.path.exists(p) else {}
 
-    Bounded sample: when a full solve to eps would exceed the budget, the oracle runs
-    a forced-k sample (eps = 0, k_s iterations, the same Alg. 1 code) and the
-    iterative-phase time is projected as (t_s / k_s) x k, with k the iteration count
-    of the full solve (the GPU's, k_hint, when given).  ``samples`` says which."""
+
+def _smt():
+    try:
+        return open("/sys/devices/system/cpu/smt/active").read().strip() == "1"
+    except Exception:
+        return None
+
+
+def run_oracle(name: str, A, b, steps: int, warmup: int, budget_s: float = 20.0, multicore: bool = False,
+               modes=("alg2", "none")):
+    """The oracle's iterative phase (Alg. 1 from the prologue to loop exit, A19), as it
+    stands, timed on the host: single thread (spcg_oracle.c) or, multicore=True, the
+    OpenMP build of the same solve phase on all cores (spcg_oracle_omp.c).
+
+    Each of warmup + steps steps is a full solve to eps when that fits the per-step
+    share of budget_s; otherwise a bounded forced-k sample (eps = 0, k_s iterations,
+    same code) whose time is projected to the oracle's OWN k to eps (oracle/kref.json,
+    one full oracle solve per config and mode) as t_s / (k_s + 1) x (k + 1)."""
     import oracle
     c = gen.CONFIGS[name]
+    kref = _kref().get(name, {})
     res = {}
-    for mode in ("alg2", "none"):
+    per_step = budget_s / len(modes) / max(steps + warmup, 1)
+    for mode in modes:
         L, U, info = oracle.setup(A, mode=mode, K=c["K"])
-        probe = oracle.pcg(A, L, U, b, 0.0, 2)                  # prologue + 2 iterations
-        per_it = probe["seconds"] / 3.0
-        k_est = (k_hint or {}).get(mode) or 100
-        if per_it * (k_est + 1) <= budget_s:
-            times, ks = [], []
-            t_start = time.perf_counter()
-            for s in range(warmup + steps):
-                r = oracle.pcg(A, L, U, b, EPS, KMAX)
-                if s >= warmup:
-                    times.append(r["seconds"] * 1e3)
-                    ks.append(r["k"])
-                if time.perf_counter() - t_start > budget_s and len(times) >= 1:
-                    break
-            res[mode] = dict(ms=float(np.mean(times)), k=int(ks[-1]), samples=len(times), projected=False,
-                             chosen_pct=info["chosen_pct"], sample=f"{len(times)} full solve(s) to eps")
+        if multicore:
+            run = lambda e, km: oracle.pcg_omp(A, L, U, b, e, km)   # noqa: E731
         else:
-            k_s = max(2, int(budget_s / per_it) - 1)
-            r = oracle.pcg(A, L, U, b, 0.0, k_s)
-            ms = r["seconds"] * 1e3 / (k_s + 1) * (k_est + 1)
-            res[mode] = dict(ms=float(ms), k=int(k_est), samples=1, projected=True, chosen_pct=info["chosen_pct"],
-                             sample=f"forced-k sample of {k_s} iterations (+ prologue), "
-                                    f"{r['seconds']:.1f} s, projected to k = {k_est}")
+            run = lambda e, km: oracle.pcg(A, L, U, b, e, km)       # noqa: E731
+        probe = run(0.0, 2)
+        per_it = probe["seconds"] / 3.0
+        threads = probe.get("threads", 1)
+        k = kref.get(mode, {}).get("k")
+        full = k is None or per_it * (k + 1) <= per_step
+        times, ks, k_s = [], [], 0
+        for sidx in range(steps + warmup):
+            if full:
+                r = run(EPS, KMAX)
+                t, kk = r["seconds"] * 1e3, r["k"]
+            else:
+                k_s = max(2, int(per_step / per_it) - 1)
+                r = run(0.0, k_s)
+                t, kk = r["seconds"] * 1e3 / (k_s + 1) * (k + 1), k
+            if sidx >= warmup:
+                times.append(t)
+                ks.append(kk)
+        sample = (f"{len(times)} full solve(s) to eps" if full else
+                  f"{len(times)} forced-k sample(s) of {k_s} iterations (+ prologue) each, projected to the "
+                  f"oracle's own k = {k} (oracle/kref.json)")
+        res[mode] = dict(ms=float(np.mean(times)), k=int(ks[-1]), samples=len(times), projected=not full,
+                         chosen_pct=info["chosen_pct"], sample=sample, threads=threads)
     return res
+
+
+def _cpu_line(name: str, o: dict, cores: int, kind_note: str) -> dict:
+    return {"value": o["alg2"]["ms"], "unit": "ms", "cores": cores, "kind": "oracle",
+            "sample": f"{name} iterative phase: {o['alg2']['sample']}, {kind_note}, {_cpu_info()}, "
+                      f"nproc {os.cpu_count()}, SMT {'on' if _smt() else 'off' if _smt() is False else '?'}; "
+                      f"PCG {o['none']['ms']:.1f} ms ({o['none']['sample']})",
+            "pcg_value": o["none"]["ms"], "iterations": o["alg2"]["k"], "pcg_iterations": o["none"]["k"],
+            "per_iter_speedup_spcg_vs_pcg": (o["none"]["ms"] / max(o["none"]["k"] + 1, 1)) /
+                                            (o["alg2"]["ms"] / max(o["alg2"]["k"] + 1, 1))}
 
 
 def main():
@@ -172,7 +209,8 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--workload", default="C2", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default=None, choices=sorted(WORKLOADS),
+                    help="default: C4 at N = 1, C5 at N > 1")
     ap.add_argument("--impl", default="spcg", choices=["spcg", "reference"])
     ap.add_argument("--sptrsv", default="auto")
     ap.add_argument("--parts", type=int, default=0)
@@ -186,7 +224,8 @@ def main():
                     help="comma list of fixed drop ratios t%% timed beside Alg. 2 and PCG (default: 1,5,10 for C4)")
     args = ap.parse_args()
     ws, rank, local = _dist()
-    name = args.workload
+    name = args.workload or ("C4" if ws == 1 else "C5")
+    args.workload = name
     if name == "C5":
         return run_batch(args, ws, rank, local)
     A = gen.config_matrix(name)
@@ -196,17 +235,16 @@ def main():
     if args.impl == "reference":
         if rank != 0:
             return
-        o = run_oracle(name, A, b, args.steps, args.warmup, budget_s=60.0)      # k: the oracle's own
+        o = run_oracle(name, A, b, args.steps, args.warmup, budget_s=150.0)
         v = o["alg2"]["ms"]
+        cpu = _cpu_line(name, o, 1, "single thread (the oracle as it stands)")
         line = {"metric": "SPCG iter-phase ms to eps=1e-8 + HBM GB/s per iter vs unsparsified PCG",
-                "impl": "reference", "value": v, "unit": "ms", "n_gpus": args.gpus, "steps": o["alg2"]["samples"],
+                "impl": "reference", "value": v, "unit": "ms", "n_gpus": args.gpus, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": v, "higher_is_better": False, "scaling": "weak",
                 "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": WORKLOADS[name], "n": A.n, "nnz": A.nnz, "K": K, "eps": EPS},
                 "iterations": o["alg2"]["k"], "pcg": {"value": o["none"]["ms"], "iterations": o["none"]["k"]},
-                "cpu_baseline": {"value": v, "unit": "ms", "cores": 1, "kind": "oracle",
-                                 "sample": f"{name} iterative phase: {o['alg2']['sample']}, single thread, "
-                                           f"{_cpu_info()}"},
+                "cpu_baseline": cpu,
                 "e2e": {"value": v, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
         print(json.dumps(line))
         return
@@ -255,11 +293,13 @@ def main():
             wall = (time.perf_counter() - t0) * 1e3
             # e2e through the public API with HOST buffers (H2D b, solve, D2H x inside the call)
             e2e = []
+            bh = torch.from_numpy(b).pin_memory()
+            xh = torch.empty_like(bh).pin_memory()
             for _ in range(max(3, args.steps // 2)):
                 flush.zero_()
                 torch.cuda.synchronize(dev)
                 te = time.perf_counter()
-                xh, info_h = h.solve_host(b, EPS, KMAX)
+                h.solve_host(bh, EPS, KMAX, out=xh)
                 e2e.append((time.perf_counter() - te) * 1e3)
             results[mode] = dict(ms=float(np.mean(ms)), ms_max=float(np.max(ms)), k=int(ks[-1]), wall=wall,
                                  e2e=float(np.mean(e2e)), info=h.info)
@@ -308,12 +348,14 @@ def main():
         l2_hit = json.load(open(os.path.join(ROOT, "profiles", "ncu_summary.json")))[name]["spcg"].get("l2_hit_pct")
     except Exception:
         pass
-    cpu = None
+    l2_resident = s_bi < 100e6
+    cpu = cpu_mc = None
     if not args.no_cpu_baseline:
-        o = run_oracle(name, A, b, 2, 0, budget_s=20.0, k_hint={"alg2": s["k"], "none": p["k"]})
-        cpu = {"value": o["alg2"]["ms"], "unit": "ms", "cores": 1, "kind": "oracle",
-               "sample": f"{name} iterative phase: {o['alg2']['sample']}, single thread, {_cpu_info()}; "
-                         f"PCG {o['none']['ms']:.1f} ms ({o['none']['sample']})"}
+        o = run_oracle(name, A, b, 1, 0, budget_s=24.0)
+        cpu = _cpu_line(name, o, 1, "single thread (the oracle as it stands)")
+        om = run_oracle(name, A, b, 1, 0, budget_s=24.0, multicore=True)
+        cpu_mc = _cpu_line(name, om, om["alg2"]["threads"], "OpenMP level-scheduled solve phase on all host cores "
+                                                            "(oracle/spcg_oracle_omp.c)")
     line = {
         "metric": "SPCG iter-phase ms to eps=1e-8 + HBM GB/s per iter vs unsparsified PCG",
         "value": s_ms, "unit": "ms", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
@@ -341,14 +383,15 @@ def main():
                                 else "spcg_pcg_kernel (persistent, whole Alg. 1)"),
                      "peak_source": peak_src,
                      "achieved_def": "B_iter (DESIGN.md §4) x iterations / CUDA-event time of the launch",
-                     "l2_hit_pct": l2_hit,
+                     "l2_hit_pct": l2_hit, "l2_resident": l2_resident,
                      "note": ("working set L2-resident (B_iter < 126 MB L2; ncu DRAM traffic << algorithmic): "
-                              "the HBM roofline is not the binding one; the chain floor is (chain_floor)"
-                              if s_bi < 100e6 else "the wavefront chain binds before HBM (chain_floor)")},
+                              "frac is algorithmic bytes over the HBM peak, not an HBM utilisation"
+                              if l2_resident else "working set >> L2: algorithmic bytes over the measured HBM peak")},
         "cpu_baseline": cpu,
+        "cpu_baseline_multicore": cpu_mc,
         "chain_floor": chain_floor(calib, si, s_bi, peak, s_ms / max(s["k"], 1)),
         "e2e": {"value": s_e2e, "unit": "ms", "h2d_bytes_per_step": 8 * A.n, "d2h_bytes_per_step": 8 * A.n,
-                "path": "spcg_solve with SPCG_HOST_PTRS (pageable host b, x)"},
+                "path": "spcg_solve with SPCG_HOST_PTRS (pinned host b, x; H2D + solve + D2H inside the call, wall clock)"},
         "gpu_launches": args.steps,
         "clocks": clocks,
         "setup_ms": {k: si[k] for k in si if k.startswith("setup_ms")},
@@ -426,34 +469,46 @@ def run_batch(args, ws, rank, local):
     sms = torch.cuda.get_device_properties(local).multi_processor_count
     hs = batch.setup_rank(plan[rank], device=local, lanes=args.lanes, sms=sms)
 
-    order = {}
+    def timed(hs_):
+        order = {}
 
-    def step():
-        if args.lanes > 1 and args.sched == "dynamic":
-            r, mk = batch.solve_rank_dynamic(hs, args.lanes, order=order or None)
-            order.update({x.index: x.iter_phase_ms for x in r})      # longest first next time
-            return r, mk
-        if args.lanes > 1:
-            return batch.solve_rank_concurrent(hs)
-        r = batch.solve_rank(hs)
-        return r, sum(x.iter_phase_ms for x in r)
+        def step():
+            if args.lanes > 1 and args.sched == "dynamic":
+                r, mk = batch.solve_rank_dynamic(hs_, args.lanes, order=order or None)
+                order.update({x.index: x.iter_phase_ms for x in r})      # longest first next time
+                return r, mk
+            if args.lanes > 1:
+                return batch.solve_rank_concurrent(hs_)
+            r = batch.solve_rank(hs_)
+            return r, sum(x.iter_phase_ms for x in r)
 
-    last = None
-    for _ in range(max(1, args.warmup)):
-        last = step()
-    if args.lanes > 1 and args.sched == "static":
-        # static lanes re-planned by LPT over the warm-up step's measured per-system times
-        batch.replan_lanes(hs, {x.index: x.iter_phase_ms for x in last[0]}, args.lanes)
-        step()
-    t_dev = []
-    clk = Clocks(local)
-    with clk:
+        last = None
+        for _ in range(max(1, args.warmup)):
+            last = step()
+        if args.lanes > 1 and args.sched == "static":
+            # static lanes re-planned by LPT over the warm-up step's measured per-system times
+            batch.replan_lanes(hs_, {x.index: x.iter_phase_ms for x in last[0]}, args.lanes)
+            step()
+        t_dev_ = []
+        res_ = None
         for _ in range(args.steps):
             torch.cuda.synchronize()
             if ws > 1:
                 torch.distributed.barrier()
-            res, mk = step()
-            t_dev.append(mk)
+            res_, mk = step()
+            t_dev_.append(mk)
+        return res_, t_dev_
+
+    clk = Clocks(local)
+    with clk:
+        res, t_dev = timed(hs)
+    # the unsparsified PCG on the same batch (metric: "... vs unsparsified PCG")
+    hs_pcg = batch.setup_rank(plan[rank], device=local, mode="none", lanes=args.lanes, sms=sms)
+    res_pcg, t_pcg = timed(hs_pcg)
+    ms_pcg = float(np.mean(t_pcg))
+    pcg_bytes = sum(h.info["algo_bytes_per_iter"] * r.iterations for (_, _, _, h, _), r in zip(hs_pcg, res_pcg))
+    for it in hs_pcg:
+        it[3].close()
     ms = float(np.mean(t_dev))
     # e2e through the public API with host buffers (H2D b, solve, D2H x inside each call)
     te = time.perf_counter()
@@ -463,12 +518,13 @@ def run_batch(args, ws, rank, local):
     bytes_rank = sum(h.info["algo_bytes_per_iter"] * r.iterations for (_, _, _, h, _), r in zip(hs, res))
     allr = batch.gather(res, ws)
     if ws > 1:
-        t = torch.tensor([ms, e2e_ms], dtype=torch.float64, device=f"cuda:{local}")
+        t = torch.tensor([ms, e2e_ms, ms_pcg], dtype=torch.float64, device=f"cuda:{local}")
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms, e2e_ms = float(t[0].item()), float(t[1].item())
-        b = torch.tensor([bytes_rank], dtype=torch.float64, device=f"cuda:{local}")
+        ms, e2e_ms, ms_pcg = float(t[0].item()), float(t[1].item()), float(t[2].item())
+        b = torch.tensor([bytes_rank, pcg_bytes], dtype=torch.float64, device=f"cuda:{local}")
         torch.distributed.all_reduce(b)
-        bytes_rank = float(b.item())
+        bytes_rank, pcg_bytes = float(b[0].item()), float(b[1].item())
+    allp = batch.gather(res_pcg, ws)
     if rank == 0:
         peak, peak_src = _peaks()
         gbs = bytes_rank / (ms * 1e-3) / 1e9
@@ -493,6 +549,10 @@ def run_batch(args, ws, rank, local):
                                        "; max over ranks",
                            "l2": "no flush: 64 different systems run back to back (working set >> L2)"},
                 "systems_per_s": len(systems) / (ms * 1e-3),
+                "pcg": {"value": ms_pcg, "unit": "ms", "hbm_gbs": pcg_bytes / (ms_pcg * 1e-3) / 1e9,
+                        "iterations_total": sum(r.iterations for r in allp),
+                        "note": "the same batch, same lanes and schedule, Ahat = A (no sparsification)"},
+                "spcg_vs_pcg": {"makespan_speedup": ms_pcg / ms},
                 "roofline": {"bound": "hbm", "achieved": gbs, "peak": peak, "unit": "GB/s", "frac": gbs / peak,
                              "traffic": None, "kernel": "spcg_pcg_kernel (one launch per system)",
                              "peak_source": peak_src,

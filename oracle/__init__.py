@@ -186,12 +186,12 @@ def ilu_numeric(Ahat: CSR, P: CSR):
     return st, _out(L, "L_s"), _out(U, "U"), -1
 
 
-def iluk(Ahat: CSR, K: int):
+def iluk(Ahat: CSR, K: int, with_levels: bool = False):
     P, lev = iluk_symbolic(Ahat, K)
     st, L, U, bad = ilu_numeric(Ahat, P)
     if st != 0:
         raise ZeroDivisionError(f"zero pivot at row {bad}")
-    return L, U
+    return (L, U, lev) if with_levels else (L, U)
 
 
 # ---------------------------------------------------------------- O9 / O10
@@ -245,6 +245,58 @@ def setup(A: CSR, mode: str = "alg2", K: int = 0, fixed_pct: float = 0.0, **alg2
         Ahat, idx, tr, wA = alg2(A, **alg2_kw)
         ratios = alg2_kw.get("ratios", (10.0, 5.0, 1.0))
         info.update(chosen_pct=ratios[idx], trace=tr, w_A=wA)
-    L, U = iluk(Ahat, K)
+    L, U, flev = iluk(Ahat, K, with_levels=True)
     info["Ahat"] = Ahat
+    info["fill_level"] = flev          # level of fill per entry of pattern(L + U), row-major (O6)
     return L, U, info
+
+
+# ---------------------------------------------------------------- multicore baseline
+_OMP_SRC = os.path.join(_HERE, "spcg_oracle_omp.c")
+_OMP_LIB = os.path.join(_HERE, "liboracle_omp.so")
+_omp = None
+
+
+def build_omp(force: bool = False) -> str:
+    if force or not os.path.exists(_OMP_LIB) or os.path.getmtime(_OMP_LIB) < os.path.getmtime(_OMP_SRC):
+        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-fPIC",
+                               "-shared", "-o", _OMP_LIB + ".tmp", _OMP_SRC, "-lm"])
+        os.replace(_OMP_LIB + ".tmp", _OMP_LIB)
+    return _OMP_LIB
+
+
+def _load_omp():
+    global _omp
+    if _omp is None:
+        lib = ctypes.CDLL(build_omp())
+        P = ctypes.c_void_p
+        CP = ctypes.POINTER(_Csr)
+        lib.or_pcg_omp.argtypes = [CP, CP, CP, P, P, ctypes.c_int64, P, P, ctypes.c_int64, P, ctypes.c_double,
+                                   ctypes.c_int64, ctypes.c_int, P, P, P, P]
+        lib.or_pcg_omp.restype = ctypes.c_int
+        lib.or_omp_threads.restype = ctypes.c_int
+        _omp = lib
+    return _omp
+
+
+def omp_threads() -> int:
+    return int(_load_omp().or_omp_threads())
+
+
+def pcg_omp(A: CSR, L: CSR, U: CSR, b: np.ndarray, eps: float, kmax: int, threads: int = 0):
+    """Algorithm 1 on all host cores (OpenMP, level-scheduled SpTRSV over the oracle's
+    own level sets).  The multicore CPU baseline (not a parity reference: reductions
+    sum in a thread-dependent order).  Returns dict(x, k, rnorm, status, seconds, threads)."""
+    wl, levl = levels_lower(L)
+    wu, levu = levels_upper(U)
+    pl, rl = level_sets(levl, wl)
+    pu, ru = level_sets(levu, wu)
+    x = np.zeros(A.n)
+    k = np.zeros(1, np.int64)
+    rn = np.zeros(1)
+    sec = np.zeros(1)
+    st = _load_omp().or_pcg_omp(ctypes.byref(_in(A)), ctypes.byref(_in(L)), ctypes.byref(_in(U)), _p(pl), _p(rl), wl,
+                                _p(pu), _p(ru), wu, _p(np.ascontiguousarray(b, np.float64)), eps, kmax, threads,
+                                _p(x), _p(k), _p(rn), _p(sec))
+    return dict(x=x, k=int(k[0]), rnorm=float(rn[0]), status=int(st), seconds=float(sec[0]),
+                threads=threads if threads > 0 else omp_threads())

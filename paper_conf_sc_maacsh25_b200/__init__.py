@@ -290,13 +290,27 @@ class SPCG:
         _check(st, "spcg_solve_wait")
         return self._solve_info(info)
 
-    def solve_host(self, b: np.ndarray, eps=1e-8, kmax=10000, x0=None):
-        """Host buffers: the library copies b (and x0) in and x out inside the call (e2e path)."""
-        b = np.ascontiguousarray(b, np.float64)
-        x = np.zeros(self.n) if x0 is None else np.ascontiguousarray(x0, np.float64).copy()
+    def solve_host(self, b, eps=1e-8, kmax=10000, x0=None, out=None):
+        """Host buffers: the library copies b (and x0) in and x out inside the call (e2e path).
+        b: numpy array or (pinned) CPU torch tensor; out: optional host buffer of the same kind
+        for x (returned)."""
+        if isinstance(b, np.ndarray):
+            b = np.ascontiguousarray(b, np.float64)
+            bp = b.ctypes.data
+            x = out if out is not None else np.zeros(self.n)
+            if x0 is not None:
+                x[:] = x0
+            xp = x.ctypes.data
+        else:                                    # CPU torch tensor (e.g. pin_memory=True)
+            assert not b.is_cuda and b.is_contiguous() and b.numel() == self.n
+            bp = b.data_ptr()
+            x = out if out is not None else _torch().zeros_like(b)
+            if x0 is not None:
+                x.copy_(_torch().as_tensor(x0))
+            xp = x.data_ptr()
         info = SolveInfo()
         flags = HOST_PTRS | (USE_X0 if x0 is not None else 0)
-        st = load().spcg_solve(self._h, b.ctypes.data, x.ctypes.data, float(eps), int(kmax), flags, ctypes.byref(info))
+        st = load().spcg_solve(self._h, bp, xp, float(eps), int(kmax), flags, ctypes.byref(info))
         _check(st, "spcg_solve")
         return x, self._solve_info(info)
 

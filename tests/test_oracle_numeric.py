@@ -256,3 +256,61 @@ def test_pcg_forced_k_and_kmax():
     assert r["k"] == 5 and r["status"] == oracle.NOT_CONVERGED
     # monotone residual history is not guaranteed for CG, but rhist[0] = ||b|| = 1
     assert r["rhist"][0] == pytest.approx(1.0, rel=1e-15)
+
+
+def test_pcg_initial_guess_branch_pins():
+    """O10's x0 branch (Alg. 1 line 2, r0 = b - A x0; A15), pinned without the oracle:
+    (a) x0 = the exact solution of a system whose b is formed exactly (small integers)
+        gives r0 = 0, so the test before the first SpMV fires: k = 0, x = x0 bitwise;
+    (b) a dense 3x3 SPD matrix: ILU(0) of a full pattern is its exact LU, so from ANY x0
+        one iteration lands on x = A^-1 b (closed form of the 3x3 inverse by Cramer's
+        rule) — a sign or operand error in r0 = b - A x0 gives a different point;
+    (c) M = I (plain CG) on a 2x2 SPD system reaches the closed-form solution in <= 2
+        iterations from x0 != 0."""
+    d = np.array([[4.0, -1.0, 0.0], [-1.0, 4.0, -1.0], [0.0, -1.0, 4.0]])
+    A = gen.from_dense(d)
+    xs = np.array([1.0, 2.0, -3.0])
+    b = d @ xs                                    # exact in fp64 (small integers)
+    L, U = oracle.iluk(A, 0)
+    r = oracle.pcg(A, L, U, b, 1e-12, 50, x0=xs)
+    assert r["k"] == 0 and r["status"] == 0 and np.array_equal(r["x"], xs)
+    # (b) dense 3x3 SPD, exact preconditioner
+    d3 = np.array([[5.0, 2.0, 1.0], [2.0, 6.0, 3.0], [1.0, 3.0, 7.0]])
+    A3 = gen.from_dense(d3)
+    L3, U3 = oracle.iluk(A3, 0)
+    b3 = np.array([1.0, -2.0, 0.5])
+    # Cramer's rule: x_i = det(A with column i replaced by b) / det(A)
+    det = np.linalg.det(d3)
+    xc = np.array([np.linalg.det(np.column_stack([b3 if c == i else d3[:, c] for c in range(3)])) / det
+                   for i in range(3)])
+    x0 = np.array([10.0, -7.0, 3.0])
+    r3 = oracle.pcg(A3, L3, U3, b3, 1e-13, 5, x0=x0)
+    assert r3["k"] == 1
+    assert np.allclose(r3["x"], xc, rtol=1e-13, atol=1e-14)
+    # (c) 2x2, M = I: CG terminates in n = 2 steps (closed-form inverse)
+    d2 = np.array([[3.0, 1.0], [1.0, 2.0]])
+    A2 = gen.from_dense(d2)
+    b2 = np.array([1.0, 1.0])
+    x2 = np.array([2.0 * 1.0 - 1.0 * 1.0, -1.0 * 1.0 + 3.0 * 1.0]) / (3.0 * 2.0 - 1.0)   # (1/5, 2/5)
+    r2 = oracle.pcg(A2, None, None, b2, 1e-14, 10, x0=np.array([-4.0, 9.0]))
+    assert r2["k"] <= 2 and r2["status"] == 0
+    assert np.allclose(r2["x"], x2, rtol=1e-14, atol=1e-15)
+
+
+def test_pcg_breakdown_branch_pin():
+    """O10's breakdown branch ((p, A p) <= 0, A12/§8(b) SPCG_ERR_BREAKDOWN): the
+    symmetric matrix [[1,2],[2,1]] has a positive diagonal but eigenvalues 3 and -1.
+    With b = (1,-1)/sqrt(2) (the -1 eigenvector) and M = I, p0 = b and
+    (p0, A p0) = -1 in closed form; with ILU(0) (= exact LU here, u_22 = -3 < 0 is
+    allowed) p0 = A^-1 b = -b and (p0, A p0) = -1 as well.  Both stop at k = 0
+    with status BREAKDOWN and x = x0 = 0."""
+    d = np.array([[1.0, 2.0], [2.0, 1.0]])
+    A = gen.from_dense(d)
+    b = np.array([1.0, -1.0]) / math.sqrt(2.0)
+    assert float(b @ d @ b) == pytest.approx(-1.0, rel=1e-15)
+    r = oracle.pcg(A, None, None, b, 1e-10, 10)
+    assert r["status"] == oracle.BREAKDOWN and r["k"] == 0 and not np.any(r["x"])
+    L, U = oracle.iluk(A, 0)
+    assert U.val[U.row_ptr[1]] == -3.0                      # negative pivot: allowed (A12)
+    r = oracle.pcg(A, L, U, b, 1e-10, 10)
+    assert r["status"] == oracle.BREAKDOWN and r["k"] == 0 and not np.any(r["x"])
