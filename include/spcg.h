@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define SPCG_ABI_VERSION 1
+#define SPCG_ABI_VERSION 2
 
 typedef int32_t spcg_status_t;
 enum {
@@ -94,10 +94,32 @@ enum {
     SPCG_SPTRSV_SYNCFREE = 2,   /* per-row ready flags, no level barriers */
     SPCG_SPTRSV_CHUNKED = 3,    /* rows partitioned into contiguous per-CTA chunks; intra-chunk
                                    dependencies through shared memory, cross-chunk through flags */
-    SPCG_SPTRSV_RESIDENT = 4    /* small systems (n <= SPCG_RESIDENT_MAX_N): one CTA holds every
+    SPCG_SPTRSV_RESIDENT = 4,   /* small systems (n <= SPCG_RESIDENT_MAX_N): one CTA holds every
                                    vector in shared memory; level-scheduled with CTA barriers */
+    SPCG_SPTRSV_WCHAIN = 5      /* warp chains: rows split into chains (decoupled components or
+                                   grid blocks), one warp walks a chain wavefront by wavefront with
+                                   register (shuffle) handoffs; vectors in execution order */
 };
 #define SPCG_RESIDENT_MAX_N 4096
+
+/* How the device loop of Algorithm 1 is orchestrated. */
+enum {
+    SPCG_EXEC_AUTO = 0,         /* = PERSISTENT */
+    SPCG_EXEC_PERSISTENT = 1,   /* one persistent cooperative kernel per solve (device-side scalars) */
+    SPCG_EXEC_GRAPH_WHILE = 2   /* a conditional-WHILE CUDA graph of per-phase kernels: NOT built in this
+                                   library (a kernel launch per wavefront or phase is the design the
+                                   persistent kernel replaces); setup returns SPCG_ERR_INVALID_ARG */
+};
+
+/* Device allocator hooks: when dev_alloc is set, every device buffer the handle owns
+ * comes from dev_alloc(bytes, stream, ctx) and goes back through
+ * dev_free(ptr, bytes, stream, ctx) (e.g. PyTorch's caching allocator; the Python
+ * binding installs such a shim).  NULL = cudaMalloc / cudaFree.  A NULL return from
+ * dev_alloc fails setup with SPCG_ERR_OOM.  The hooks are called from the thread that
+ * calls spcg_setup / spcg_solve / spcg_destroy, never from device code, and must stay
+ * valid (with ctx) until spcg_destroy returns. */
+typedef void* (*spcg_dev_alloc_fn)(size_t bytes, void* stream, void* ctx);
+typedef void (*spcg_dev_free_fn)(void* ptr, size_t bytes, void* stream, void* ctx);
 
 typedef struct {
     int32_t device;             /* CUDA ordinal; -1 = host analysis only (export works, solve does not) */
@@ -105,7 +127,15 @@ typedef struct {
     int32_t sptrsv;             /* SPCG_SPTRSV_* */
     int32_t parts;              /* CTAs of the persistent kernel (0 = auto from n and the SM count) */
     int32_t host_threads;       /* OpenMP threads for setup (0 = all) */
-    int32_t reserved[8];
+    int32_t exec;               /* SPCG_EXEC_* */
+    spcg_dev_alloc_fn dev_alloc;
+    spcg_dev_free_fn dev_free;
+    void* alloc_ctx;
+    double wide_min;            /* mean dependencies per row above which LEVEL/SYNCFREE use one warp per
+                                   row (0 = default SPCG_WCAP = 8) */
+    int32_t chunk_partition;    /* CHUNKED executor: -1 = inspector's choice (default), else force
+                                   0 contiguous, 1 strided, 2 affinity, 3 components, 4 tiles */
+    int32_t reserved[7];
 } spcg_options_t;
 
 typedef struct {
@@ -130,7 +160,11 @@ typedef struct {
     double algo_bytes_per_iter; /* B_iter: what one iteration must move */
     double algo_flops_per_iter;
     int32_t partition;          /* CHUNKED: row partition the inspector chose — 0 contiguous, 1 strided,
-                                   2 affinity, 3 components, 4 tiles; -1 otherwise */
+                                   2 affinity, 3 components, 4 tiles; WCHAIN: 5
+                                   components, 6 grid3d, 7 grid2d; -1 otherwise */
+    int32_t chains;             /* WCHAIN: warp chains (0 otherwise) */
+    int64_t positions;          /* WCHAIN: execution-order slots (32 x steps >= n) */
+    int64_t chain_entries[4];   /* WCHAIN: dependencies read by shuffle / shared ring / global / flag */
 } spcg_setup_info_t;
 
 typedef struct {

@@ -27,7 +27,10 @@ ERR_INVALID_ARG, ERR_BAD_MATRIX, ERR_ZERO_PIVOT, ERR_BREAKDOWN = -1, -2, -3, -4
 ERR_OOM, ERR_CUDA, ERR_INTERNAL, ERR_NO_DEVICE = -5, -6, -7, -8
 
 DROP_NONE, DROP_FIXED, DROP_WAVEFRONT_AWARE = 0, 1, 2
-SPTRSV = {"auto": 0, "level": 1, "syncfree": 2, "chunked": 3, "resident": 4}
+SPTRSV = {"auto": 0, "level": 1, "syncfree": 2, "chunked": 3, "resident": 4, "wchain": 5}
+EXEC = {"auto": 0, "persistent": 1, "graph_while": 2}
+PARTITION_NAME = {0: "contiguous", 1: "strided", 2: "affinity", 3: "components", 4: "tiles",
+                  5: "chain-components", 6: "chain-grid3d", 7: "chain-grid2d"}
 RESIDENT_MAX_N = 4096          # include/spcg.h SPCG_RESIDENT_MAX_N
 SPTRSV_NAME = {v: k for k, v in SPTRSV.items()}
 USE_X0, HOST_PTRS = 0x1, 0x2
@@ -35,12 +38,17 @@ USE_X0, HOST_PTRS = 0x1, 0x2
 EXPORT = dict(ahat_rowptr=1, ahat_col=2, ahat_val=3, l_rowptr=4, l_col=5, l_val=6, u_rowptr=7, u_col=8,
               u_val=9, fill_level=10, level_l=11, level_u=12, levelptr_l=13, levelrows_l=14,
               levelptr_u=15, levelrows_u=16, rhist=17, dbg_stream=100, dbg_part_chunk=101, dbg_part_uchunk=102,
-              dbg_part_begin=103)
+              dbg_part_begin=103, dbg_chain_recl=104, dbg_chain_recu=105, dbg_chain_perm=106,
+              dbg_chain_step=107, dbg_chain_flags=108, dbg_chain_a_eoff=109, dbg_chain_a_col=110,
+              dbg_chain_a_val=111)
 _EXPORT_DT = dict(ahat_rowptr=np.int64, ahat_col=np.int32, ahat_val=np.float64, l_rowptr=np.int64,
                   l_col=np.int32, l_val=np.float64, u_rowptr=np.int64, u_col=np.int32, u_val=np.float64,
                   fill_level=np.int32, level_l=np.int32, level_u=np.int32, levelptr_l=np.int64,
                   levelrows_l=np.int32, levelptr_u=np.int64, levelrows_u=np.int32, rhist=np.float64,
-                  dbg_stream=np.uint8, dbg_part_chunk=np.int32, dbg_part_uchunk=np.int32, dbg_part_begin=np.int64)
+                  dbg_stream=np.uint8, dbg_part_chunk=np.int32, dbg_part_uchunk=np.int32, dbg_part_begin=np.int64,
+                  dbg_chain_recl=np.uint8, dbg_chain_recu=np.uint8, dbg_chain_perm=np.int32, dbg_chain_step=np.int64,
+                  dbg_chain_flags=np.uint32, dbg_chain_a_eoff=np.int64, dbg_chain_a_col=np.int32,
+                  dbg_chain_a_val=np.float64)
 
 
 class SpcgError(RuntimeError):
@@ -60,9 +68,16 @@ class DropParams(ctypes.Structure):
                 ("norm_reading", ctypes.c_int32), ("reduction_denominator", ctypes.c_int32)]
 
 
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+
+
 class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("stream", ctypes.c_void_p), ("sptrsv", ctypes.c_int32),
-                ("parts", ctypes.c_int32), ("host_threads", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
+                ("parts", ctypes.c_int32), ("host_threads", ctypes.c_int32), ("exec", ctypes.c_int32),
+                ("dev_alloc", _ALLOC_FN), ("dev_free", _FREE_FN), ("alloc_ctx", ctypes.c_void_p),
+                ("wide_min", ctypes.c_double), ("chunk_partition", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 7)]
 
 
 class SetupInfo(ctypes.Structure):
@@ -77,7 +92,8 @@ class SetupInfo(ctypes.Structure):
                 ("setup_ms_layout", ctypes.c_double), ("setup_ms_upload", ctypes.c_double),
                 ("sptrsv", ctypes.c_int32), ("parts", ctypes.c_int32), ("device_bytes", ctypes.c_int64),
                 ("algo_bytes_per_iter", ctypes.c_double), ("algo_flops_per_iter", ctypes.c_double),
-                ("partition", ctypes.c_int32)]
+                ("partition", ctypes.c_int32), ("chains", ctypes.c_int32), ("positions", ctypes.c_int64),
+                ("chain_entries", ctypes.c_int64 * 4)]
 
 
 class SolveInfo(ctypes.Structure):
@@ -134,7 +150,7 @@ def load(path: str | None = None):
     lib.spcg_set_stream.restype = I32
     lib.spcg_calibrate.argtypes = [I32, ctypes.POINTER(Calib)]
     lib.spcg_calibrate.restype = I32
-    if lib.spcg_abi_version() != 1:
+    if lib.spcg_abi_version() != 2:
         raise ImportError("libspcg ABI version mismatch")
     _lib = lib
     return lib
@@ -183,11 +199,44 @@ def _torch():
     return torch
 
 
+class _TorchAllocator:
+    """spcg_options_t.dev_alloc / dev_free backed by PyTorch's caching allocator, so the
+    library's device buffers are owned by torch (north_star: PyTorch provides device
+    memory and streams).  The ctypes callbacks are kept alive by the handle."""
+
+    def __init__(self, device: int):
+        torch = _torch()
+        self.device = device
+        self.live = {}
+
+        def _alloc(nbytes, stream, ctx):
+            try:
+                ptr = torch.cuda.caching_allocator_alloc(int(nbytes), self.device, int(stream or 0))
+            except Exception:          # OOM: the library reports SPCG_ERR_OOM
+                return None
+            self.live[ptr] = nbytes
+            return ptr
+
+        def _free(ptr, nbytes, stream, ctx):
+            if ptr in self.live:
+                del self.live[ptr]
+                try:
+                    torch.cuda.caching_allocator_delete(ptr)
+                except Exception:      # interpreter shutdown: the process frees the device memory
+                    pass
+
+        self.alloc_fn = _ALLOC_FN(_alloc)
+        self.free_fn = _FREE_FN(_free)
+
+
 class SPCG:
-    """A set-up SPCG preconditioner + solver bound to one device (or host-only, device=-1)."""
+    """A set-up SPCG preconditioner + solver bound to one device (or host-only, device=-1).
+
+    allocator: "torch" (default: device buffers from PyTorch's caching allocator through
+    the spcg_options_t hooks) or "cuda" (the library's own cudaMalloc)."""
 
     def __init__(self, A, mode="alg2", K=0, fixed_pct=0.0, sptrsv="auto", parts=0, device=0, stream=None,
-                 host_threads=0, **drop_kw):
+                 host_threads=0, allocator="torch", exec="auto", wide_min=0.0, chunk_partition=-1, **drop_kw):
         lib = load()
         rp = np.ascontiguousarray(A.row_ptr, np.int64)
         col = np.ascontiguousarray(A.col, np.int32)
@@ -201,13 +250,21 @@ class SPCG:
         opt.sptrsv = SPTRSV[sptrsv] if isinstance(sptrsv, str) else int(sptrsv)
         opt.parts = parts
         opt.host_threads = host_threads
+        opt.exec = EXEC[exec]
+        opt.wide_min = wide_min
+        opt.chunk_partition = chunk_partition
         self.device = device
+        self._alloc = None
         if device >= 0:
             torch = _torch()
             if stream is None:
                 stream = torch.cuda.current_stream(device)
             self.stream = stream
             opt.stream = stream.cuda_stream
+            if allocator == "torch":
+                self._alloc = _TorchAllocator(device)
+                opt.dev_alloc = self._alloc.alloc_fn
+                opt.dev_free = self._alloc.free_fn
         h = ctypes.c_void_p()
         _check(lib.spcg_setup(ctypes.byref(c), ctypes.byref(dp), K, ctypes.byref(opt), ctypes.byref(h)), "spcg_setup")
         self._h = h
@@ -216,8 +273,7 @@ class SPCG:
         self.info = {f[0]: (list(getattr(si, f[0])) if isinstance(getattr(si, f[0]), ctypes.Array)
                             else getattr(si, f[0])) for f in SetupInfo._fields_}
         self.info["sptrsv_name"] = SPTRSV_NAME.get(self.info["sptrsv"], "?")
-        self.info["partition_name"] = {0: "contiguous", 1: "strided", 2: "affinity", 3: "components", 4: "tiles"}.get(
-            self.info["partition"], "-")
+        self.info["partition_name"] = PARTITION_NAME.get(self.info["partition"], "-")
 
     def close(self):
         h = getattr(self, "_h", None)

@@ -91,6 +91,12 @@ void spcg_options_default(spcg_options_t* o) {
     o->sptrsv = SPCG_SPTRSV_AUTO;
     o->parts = 0;
     o->host_threads = 0;
+    o->exec = SPCG_EXEC_AUTO;
+    o->dev_alloc = nullptr;
+    o->dev_free = nullptr;
+    o->alloc_ctx = nullptr;
+    o->wide_min = 0.0;
+    o->chunk_partition = -1;
 }
 
 int spcg_dev_sm_count(int device);   // kernels.cu
@@ -109,6 +115,15 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
     if (drop.mode < 0 || drop.mode > 2) { set_error("bad drop mode"); return SPCG_ERR_INVALID_ARG; }
     spcg_options_t opt;
     if (opt_in) opt = *opt_in; else spcg_options_default(&opt);
+    if (opt.exec == SPCG_EXEC_GRAPH_WHILE) {
+        set_error("exec GRAPH_WHILE is not built: the iterative phase runs as one persistent kernel");
+        return SPCG_ERR_INVALID_ARG;
+    }
+    if (opt.exec < 0 || opt.exec > SPCG_EXEC_GRAPH_WHILE) { set_error("bad exec"); return SPCG_ERR_INVALID_ARG; }
+    if ((opt.dev_alloc == nullptr) != (opt.dev_free == nullptr)) {
+        set_error("dev_alloc and dev_free must be given together");
+        return SPCG_ERR_INVALID_ARG;
+    }
 #ifdef _OPENMP
     if (opt.host_threads > 0) omp_set_num_threads(opt.host_threads);
 #endif
@@ -155,6 +170,22 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         // iteration: chunked 31.5 ms, level warp-per-row 6.3 ms, sync-free warp-per-row
         // 2.2 ms).
         int strategy = opt.sptrsv;
+        // AUTO: the warp-chain executor whenever it applies (narrow rows, a chain
+        // partition exists): every wavefront handoff inside a chain is a register
+        // shuffle; otherwise the round-1 choice below.
+        std::string chain_why;
+        bool chain_built = false;
+        if ((strategy == SPCG_SPTRSV_AUTO || strategy == SPCG_SPTRSV_WCHAIN) && !h->identity) {
+            // components are packed onto as many chains as there are SMs (or the CTAs asked for)
+            const int target = opt.parts > 0 ? opt.parts : (opt.device >= 0 ? spcg_dev_sm_count(opt.device) : 148);
+            chain_built = build_chain_layout(h->A, h->F, std::max(1, target), h->lay.C, &chain_why);
+            if (chain_built) strategy = SPCG_SPTRSV_WCHAIN;
+            else if (strategy == SPCG_SPTRSV_WCHAIN) {
+                delete h;
+                set_error("warp-chain executor does not apply: " + chain_why);
+                return SPCG_ERR_INVALID_ARG;
+            }
+        }
         if (strategy == SPCG_SPTRSV_AUTO) {
             const double wl = h->n > 0 ? (double)h->F.L.nnz() / (double)h->n : 0.0;
             strategy = (h->identity || wl <= (double)SPCG_WCAP) ? SPCG_SPTRSV_CHUNKED : SPCG_SPTRSV_SYNCFREE;
@@ -166,7 +197,7 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             if (!h->identity && wl <= (double)SPCG_WCAP && h->n <= SPCG_RESIDENT_MAX_N)
                 strategy = SPCG_SPTRSV_RESIDENT;
         }
-        if (strategy < 1 || strategy > 4) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }
+        if (strategy < 1 || strategy > 5) { delete h; set_error("bad sptrsv executor"); return SPCG_ERR_INVALID_ARG; }
         if (strategy == SPCG_SPTRSV_RESIDENT && h->n > SPCG_RESIDENT_MAX_N) {
             delete h;
             set_error("the resident executor holds every vector in one CTA's shared memory: n <= SPCG_RESIDENT_MAX_N");
@@ -187,14 +218,46 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             else parts = (h->n <= 4096 || h->identity) ? 1 : std::min(16, slots);
         }
         if (strategy == SPCG_SPTRSV_RESIDENT) parts = 1;
-        parts = std::max(1, std::min<int>(parts, slots));
-        if ((int64_t)parts > h->n) parts = (int)h->n;
-        build_spmv_layout(h->A, h->lay.A);
-        build_tri_layouts(h->F, strategy, parts, spcg_dev_ring_max(), h->lay);
+        if (strategy == SPCG_SPTRSV_WCHAIN) {
+            // CTAs: one per chain up to the SM count (more chains share CTAs, one solver warp
+            // each); large systems take every SM so the SpMV and vector phases use them all
+            const int nch = h->lay.C.nchains;
+            const int64_t npos = 32 * h->lay.C.nsteps;
+            if (opt.parts <= 0) parts = (nch >= slots || npos >= (1 << 17)) ? slots : nch;
+            parts = std::max(1, std::min<int>(parts, slots));
+            if ((nch + parts - 1) / parts > 8) {
+                parts = std::min(slots, (nch + 7) / 8);
+                if ((nch + parts - 1) / parts > 8) {
+                    delete h;
+                    set_error("warp-chain executor: more than 8 chains per CTA");
+                    return SPCG_ERR_INVALID_ARG;
+                }
+            }
+        } else {
+            parts = std::max(1, std::min<int>(parts, slots));
+            if ((int64_t)parts > h->n) parts = (int)h->n;
+        }
+        if (strategy != SPCG_SPTRSV_WCHAIN) {
+            h->lay.C = ChainLayout();
+            build_spmv_layout(h->A, h->lay.A);
+        }
+        if (strategy == SPCG_SPTRSV_WCHAIN) {
+            // the warp-chain kernel reads only lay.C (its own SpMV layout and records)
+            h->lay.strategy = strategy;
+            h->lay.parts = parts;
+            h->lay.ring = 0;
+            h->lay.part_begin.assign({0, h->n});
+        } else {
+            build_tri_layouts(h->F, strategy, parts, spcg_dev_ring_max(), opt.wide_min, opt.chunk_partition, h->lay);
+        }
         double t5 = now_ms();
         int64_t bytes = 0;
         if (opt.device >= 0) {
-            st = spcg_dev_create(opt.device, opt.stream, h->lay, h->n, h->identity, &h->dev, &bytes);
+            DevAllocator alc;
+            alc.alloc = opt.dev_alloc;
+            alc.free = opt.dev_free;
+            alc.ctx = opt.alloc_ctx;
+            st = spcg_dev_create(opt.device, opt.stream, h->lay, h->n, h->identity, alc, &h->dev, &bytes);
             if (st != SPCG_OK) { delete h; return st; }
         }
         double t6 = now_ms();
@@ -231,7 +294,18 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         {
             static const char* kinds[] = {"contiguous", "strided", "affinity", "components", "tiles"};
             I.partition = -1;
-            for (int k = 0; k < 5; ++k) if (h->lay.partition == kinds[k]) I.partition = k;
+            if (strategy == SPCG_SPTRSV_CHUNKED)
+                for (int k = 0; k < 5; ++k) if (h->lay.partition == kinds[k]) I.partition = k;
+            if (strategy == SPCG_SPTRSV_WCHAIN) {
+                static const char* ck[] = {"components", "grid3d", "grid2d"};
+                for (int k = 0; k < 3; ++k) if (h->lay.C.partition == ck[k]) I.partition = 5 + k;
+                I.chains = h->lay.C.nchains;
+                I.positions = 32 * h->lay.C.nsteps;
+                I.chain_entries[0] = h->lay.C.prev_entries;
+                I.chain_entries[1] = h->lay.C.hist_entries;
+                I.chain_entries[2] = h->lay.C.glob_entries;
+                I.chain_entries[3] = h->lay.C.ext_entries;
+            }
         }
         // B_iter: 12 B per stored entry of A, L_s, U_s; 1/u_ii; three row
         // pointers; two level_rows arrays; 120 B of vector traffic per row.
@@ -386,6 +460,14 @@ spcg_status_t spcg_export(spcg_handle_t h, int32_t what, void* buf, size_t* byte
         case 101: return put(h->lay.S.part_chunk, buf, bytes);
         case 102: return put(h->lay.S.part_uchunk, buf, bytes);
         case 103: return put(h->lay.part_begin, buf, bytes);
+        case 104: return put(h->lay.C.recL, buf, bytes);           // debug: warp-chain records
+        case 105: return put(h->lay.C.recU, buf, bytes);
+        case 106: return put(h->lay.C.perm, buf, bytes);
+        case 107: return put(h->lay.C.chain_step, buf, bytes);
+        case 108: return put(h->lay.C.chain_flags, buf, bytes);
+        case 109: return put(h->lay.C.A.eoff, buf, bytes);
+        case 110: return put(h->lay.C.A.col, buf, bytes);
+        case 111: return put(h->lay.C.A.val, buf, bytes);
         default: set_error("unknown export item"); return SPCG_ERR_INVALID_ARG;
     }
 }

@@ -23,7 +23,7 @@ constexpr int NWARP = BLOCK / 32;
 constexpr long long SPIN_TIMEOUT_CYC = 8ll * 1000 * 1000 * 1000;            // ~4 s of SM cycles: abort, never hang
 
 enum { ST_LEVEL = SPCG_SPTRSV_LEVEL, ST_SYNCFREE = SPCG_SPTRSV_SYNCFREE, ST_CHUNKED = SPCG_SPTRSV_CHUNKED,
-       ST_RESIDENT = SPCG_SPTRSV_RESIDENT };
+       ST_RESIDENT = SPCG_SPTRSV_RESIDENT, ST_WCHAIN = SPCG_SPTRSV_WCHAIN };
 enum { K_APPLY = 0, K_PRO = 1, K_ITER = 2 };
 enum { M_SOLVE = 0, M_SPMV = 1, M_LOWER = 2, M_UPPER = 3, M_PRECOND = 4 };
 
@@ -66,6 +66,24 @@ struct Scal {
     unsigned dbg_want, dbg_seen;
 };
 
+// warp-chain executor (wchain.cu; layout: chain_layout.cpp, internal.h ChainLayout)
+struct DevChain {
+    int32_t nchains, per_cta;      // chains, solver warps per CTA (chain c -> CTA c % grid, warp c / grid)
+    int32_t C, nst;                // steps per stage (chunk), stages per solver warp
+    int32_t W_L, W_U, rec_L, rec_U;
+    int32_t any_ext, any_hist;
+    uint32_t stage_bytes, warp_bytes, ext_off, hist_off;
+    int64_t nsteps, npos;
+    const int64_t* chain_step;     // [nchains+1]
+    const uint32_t* chain_flags;   // [nchains] CC_*
+    const uint8_t* recL;
+    const uint8_t* recU;
+    const int32_t* perm;           // [npos] row at each position, -1 padding
+    double* xp;                    // x in position order
+    double* bp;                    // b (or the apply-mode input) in position order
+    double* t1;                    // apply-mode temporary (position order)
+};
+
 struct Params {
     int64_t n;
     int ring;
@@ -100,6 +118,7 @@ struct Params {
     long long rhist_cap;
     unsigned long long* trace;     // debug timeline (env SPCG_TRACE), see trace_mark
     unsigned long long* hb;        // debug heartbeats [parts][8] (env SPCG_TRACE), see hbeat
+    DevChain CH;
 };
 // heartbeat: role slot of this CTA <- (iteration << 40) | (phase step << 20) | value
 __device__ __forceinline__ void hbeat(const Params& P, int role, unsigned long long v) {
@@ -269,12 +288,12 @@ __device__ void global_sums(const double* partials, int slot_a, int slot_b, doub
 // gathers of p, then the FMA chains (k ascending per row, as the definition):
 // SU x SK independent loads in flight instead of one dependent chain.
 constexpr int SU = 4, SK = 4;
-__device__ void phase_spmv(const Params& P, const double* pin, double* wout, double& pw) {
+__device__ void phase_spmv(const DevA& A, int64_t nrows, const double* pin, double* wout, double& pw) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int64_t ns = P.A.nslices;
+    const int64_t ns = A.nslices;
     const int64_t stride = (int64_t)gridDim.x * NWARP * SU;
     for (int64_t s0 = ((int64_t)blockIdx.x * NWARP + warp) * SU; s0 < ns; s0 += stride) {
-        const int64_t eo = (lane <= SU && s0 + lane <= ns) ? __ldg(P.A.eoff + s0 + lane) : 0;
+        const int64_t eo = (lane <= SU && s0 + lane <= ns) ? __ldg(A.eoff + s0 + lane) : 0;
         int64_t e[SU];
         int wd[SU];
         int wmax = 0;
@@ -297,8 +316,8 @@ __device__ void phase_spmv(const Params& P, const double* pin, double* wout, dou
                 for (int k = 0; k < SK; ++k) {
                     const bool on = kb + k < wd[u];
                     const int64_t idx = (e[u] + kb + k) * 32 + lane;
-                    c[u][k] = on ? __ldg(P.A.col + idx) : 0;
-                    v[u][k] = on ? __ldg(P.A.val + idx) : 0.0;
+                    c[u][k] = on ? __ldg(A.col + idx) : 0;
+                    v[u][k] = on ? __ldg(A.val + idx) : 0.0;
                 }
 #pragma unroll
             for (int u = 0; u < SU; ++u)
@@ -313,7 +332,7 @@ __device__ void phase_spmv(const Params& P, const double* pin, double* wout, dou
 #pragma unroll
         for (int u = 0; u < SU; ++u) {
             const int64_t row = (s0 + u) * 32 + lane;
-            if (s0 + u < ns && row < P.n) {
+            if (s0 + u < ns && row < nrows) {
                 wout[row] = acc[u];
                 pw = fma(pin[row], acc[u], pw);
             }

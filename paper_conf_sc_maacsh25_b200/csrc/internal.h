@@ -131,6 +131,47 @@ struct ChunkStream {
     int64_t records = 0;
 };
 
+// Warp-chain executor.  Rows are split into chains; a chain is
+// walked by one warp in steps of <= 32 rows (one per lane) of one wavefront level,
+// levels ascending (L) and the same steps in reverse (U: the reverse of a topological
+// order of L is one of U, the ILU(K) pattern being symmetric).  All vectors of
+// Algorithm 1 live in execution ("position") order pos = 32 * global_step + lane for
+// the whole solve; b and x are permuted on entry and exit.  A record per step holds,
+// per lane, W dependency tags + values (and 1/u_ii for U):
+//   tag u32: kind << 29 | payload
+//     PAD  (0): no entry (value 0)
+//     PREV (1): the value lane `payload & 31` produced in the chain's previous step
+//               (a warp shuffle, no memory access)
+//     HIST (2): lane payload & 31, `(payload >> 5) & 255` steps back (shared-memory ring)
+//     GLOB (3): own chain, older than the ring: position payload, read from global
+//     EXT  (4): another chain: position payload & (2^28-1), ordinal (payload >> 28) & 1
+//               of the lane's prefetched flags (ready flag prefetched one chunk ahead)
+//     EXTS (5): another chain, beyond two per lane and step: polled at use
+//   trailer: u32 publish mask (lanes whose value another chain reads), u32 flags.
+enum { CT_PAD = 0, CT_PREV = 1, CT_HIST = 2, CT_GLOB = 3, CT_EXT = 4, CT_EXTS = 5 };
+enum { CS_SLOW = 1, CS_EXT = 2 };                 // record trailer flags
+enum { CC_LHIST = 1, CC_LEXT = 2, CC_UHIST = 4, CC_UEXT = 8 };   // per-chain flags
+constexpr int SPCG_CHAIN_WMAX = 16;              // dependency columns per record (wider: other executors)
+constexpr int SPCG_CHAIN_HIST = 32;              // steps kept in the per-warp history ring
+
+struct ChainLayout {
+    int32_t nchains = 0;
+    int32_t W_L = 0, W_U = 0;
+    int32_t rec_L = 0, rec_U = 0;         // bytes per record
+    int64_t nsteps = 0;                   // global steps; positions = 32 * nsteps
+    std::vector<int64_t> chain_step;      // [nchains+1] first global step of each chain
+    std::vector<uint32_t> chain_flags;    // [nchains] CC_*
+    std::vector<int32_t> perm;            // [npos] row at each position (-1 padding)
+    std::vector<int32_t> iperm;           // [n] position of each row
+    std::vector<uint8_t> recL, recU;      // nsteps records each
+    SpmvLayout A;                         // SELL-32 of A over positions (slice = step)
+    std::string partition;                // components / grid2d / grid3d
+    int64_t ext_entries = 0, hist_entries = 0, glob_entries = 0, prev_entries = 0;
+};
+// Builds the chain layout when the factors suit it (dependency columns <= WMAX, a
+// partition into chains found); returns false (why set) otherwise.
+bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, ChainLayout& out, std::string* why);
+
 struct Layouts {
     int32_t strategy = SPCG_SPTRSV_LEVEL;
     int32_t parts = 1;
@@ -140,10 +181,12 @@ struct Layouts {
     SpmvLayout A;
     TriLayout L, U;
     ChunkStream S;                 // chunked executor only
+    ChainLayout C;                 // warp-chain executor only
 };
 
 void build_spmv_layout(const Csr& A, SpmvLayout& out);
-void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, Layouts& out);
+void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, double wide_min, int force_part,
+                       Layouts& out);
 
 }  // namespace spcg
 
@@ -151,8 +194,14 @@ void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, 
 struct spcg_device_s;
 typedef struct spcg_device_s spcg_device_t;
 
+struct DevAllocator {               // spcg_options_t allocator hooks (NULL: cudaMalloc / cudaFree)
+    spcg_dev_alloc_fn alloc = nullptr;
+    spcg_dev_free_fn free = nullptr;
+    void* ctx = nullptr;
+};
 spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay, int64_t n,
-                              bool identity_precond, spcg_device_t** out, int64_t* bytes);
+                              bool identity_precond, const DevAllocator& alloc, spcg_device_t** out,
+                              int64_t* bytes);
 void spcg_dev_destroy(spcg_device_t* d);
 spcg_status_t spcg_dev_solve(spcg_device_t* d, const double* b, double* x, double eps, int64_t kmax,
                              bool use_x0, spcg_solve_info_t* info, std::vector<double>* rhist);

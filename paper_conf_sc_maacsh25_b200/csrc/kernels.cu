@@ -1315,7 +1315,7 @@ __device__ __forceinline__ void pcg_body(const Params& P, double* dyn) {
     if (P.mode != M_SOLVE) {
         double a = 0.0, b = 0.0;
         if (P.mode == M_SPMV) {
-            phase_spmv(P, P.in, P.out, a);
+            phase_spmv(P.A, P.n, P.in, P.out, a);
         } else if (P.mode == M_LOWER) {
             tri_solve<STRAT>(P, 1, K_APPLY, P.in, P.out, nullptr, nullptr, nullptr, P.epoch, 0.0, a, b, ring, gen, CS, ps);
         } else if (P.mode == M_UPPER) {
@@ -1339,7 +1339,7 @@ __device__ __forceinline__ void pcg_body(const Params& P, double* dyn) {
     const double* r_src = P.b;
     if (P.use_x0) {
         double dummy = 0.0;
-        phase_spmv(P, P.x, P.w, dummy);
+        phase_spmv(P.A, P.n, P.x, P.w, dummy);
         grid_sync(P.sc, gen);
         const int64_t stride = (int64_t)gridDim.x * BLOCK;
         for (int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x; i < P.n; i += stride) P.r[i] = P.b[i] - P.w[i];
@@ -1367,7 +1367,7 @@ __device__ __forceinline__ void pcg_body(const Params& P, double* dyn) {
         if (blockIdx.x == 0 && threadIdx.x == 0) trace_mark(P, k, 0);
         // line 9-10: w = A p, sigma = (p, w), alpha = rho / sigma
         double pw = 0.0;
-        phase_spmv(P, P.p, P.w, pw);
+        phase_spmv(P.A, P.n, P.p, P.w, pw);
         block_partials(pw, 0.0, P.partials, 2, -1);
         grid_sync(P.sc, gen);
         double sigma, unused;
@@ -1460,7 +1460,9 @@ struct spcg_device_s {
     int parts = 1;
     size_t smem = 0;
     Params P{};
-    std::vector<void*> allocs;
+    DevAllocator A{};                                 // caller's allocator hooks (or cudaMalloc)
+    std::vector<std::pair<void*, size_t>> allocs;
+    size_t mb_bytes = 0;                              // bytes of each ready-flag array (mbL, mbU)
     int64_t bytes = 0;
     unsigned epoch = 1;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -1487,26 +1489,49 @@ extern "C" int spcg_dbg_heartbeats(void* handle_dev, unsigned long long* out, in
     return m;
 }
 
+// every device buffer of a handle: the caller's hooks (spcg_options_t.dev_alloc, e.g. the
+// PyTorch caching allocator) or cudaMalloc; sizes rounded up to 256 B
+static spcg_status_t dev_malloc(spcg_device_t* d, size_t b, void** out) {
+    b = (std::max<size_t>(b, 16) + 255) & ~(size_t)255;
+    void* p = nullptr;
+    if (d->A.alloc) {
+        p = d->A.alloc(b, (void*)d->stream, d->A.ctx);
+        if (!p) { spcg::set_error("dev_alloc hook returned NULL"); return SPCG_ERR_OOM; }
+    } else {
+        cudaError_t e = cudaMalloc(&p, b);
+        if (e != cudaSuccess) {
+            spcg::set_error(std::string("cudaMalloc: ") + cudaGetErrorString(e));
+            return e == cudaErrorMemoryAllocation ? SPCG_ERR_OOM : SPCG_ERR_CUDA;
+        }
+    }
+    d->allocs.push_back({p, b});
+    d->bytes += (int64_t)b;
+    *out = p;
+    return SPCG_OK;
+}
+
+static void dev_free(spcg_device_t* d, void* p) {
+    for (size_t i = 0; i < d->allocs.size(); ++i)
+        if (d->allocs[i].first == p) {
+            if (d->A.free) d->A.free(p, d->allocs[i].second, (void*)d->stream, d->A.ctx);
+            else cudaFree(p);
+            d->bytes -= (int64_t)d->allocs[i].second;
+            d->allocs.erase(d->allocs.begin() + i);
+            return;
+        }
+}
+
 template <class T>
 static spcg_status_t upload(spcg_device_t* d, const std::vector<T>& v, const T** out) {
     void* p = nullptr;
-    size_t b = std::max<size_t>(v.size() * sizeof(T), 16);
-    CK(cudaMalloc(&p, b));
-    d->allocs.push_back(p);
-    d->bytes += (int64_t)b;
+    spcg_status_t s = dev_malloc(d, v.size() * sizeof(T), &p);
+    if (s != SPCG_OK) return s;
     if (!v.empty()) CK(cudaMemcpyAsync(p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice, d->stream));
     *out = (const T*)p;
     return SPCG_OK;
 }
 
-static spcg_status_t alloc(spcg_device_t* d, size_t b, void** out) {
-    void* p = nullptr;
-    CK(cudaMalloc(&p, std::max<size_t>(b, 16)));
-    d->allocs.push_back(p);
-    d->bytes += (int64_t)b;
-    *out = p;
-    return SPCG_OK;
-}
+static spcg_status_t alloc(spcg_device_t* d, size_t b, void** out) { return dev_malloc(d, b, out); }
 
 #define UP(vec, dst)                                           \
     do {                                                       \
@@ -1553,8 +1578,11 @@ extern "C" int spcg_dev_sm_count(int device) {
 template <int STRAT>
 static void* kernel_ptr() { return (void*)spcg_pcg_kernel<STRAT>; }
 
+void* spcg_wchain_kernel_ptr();   // wchain.cu
+
 static void* pick_kernel(int strategy) {
     switch (strategy) {
+        case ST_WCHAIN: return spcg_wchain_kernel_ptr();
         case ST_RESIDENT: return (void*)spcg_resident_kernel;
         case ST_LEVEL: return kernel_ptr<ST_LEVEL>();
         case ST_SYNCFREE: return kernel_ptr<ST_SYNCFREE>();
@@ -1562,8 +1590,42 @@ static void* pick_kernel(int strategy) {
     }
 }
 
+// WCHAIN shared memory per solver warp: mbarriers, NST stages of C steps (records + the
+// pass's operand slices), the prefetched-flag queue, the history ring.  The largest
+// (C, NST) whose per-CTA total fits.
+static bool chain_smem_config(const spcg::ChainLayout& CL, int per_cta, DevChain& D, size_t* total) {
+    const size_t step_bytes = std::max<size_t>((size_t)CL.rec_L + 4 * 256, (size_t)CL.rec_U + 2 * 256);
+    const bool any_ext = CL.ext_entries > 0, any_hist = CL.hist_entries > 0;
+    static const int cfg[][2] = {{8, 4}, {8, 3}, {4, 4}, {4, 3}, {4, 2}, {2, 2}, {1, 2}};
+    const size_t limit = 227 * 1024 - 2048;       // dynamic smem per CTA, minus the static blocks
+    for (auto& cn : cfg) {
+        const int C = cn[0], NST = cn[1];
+        const size_t stage = (C * step_bytes + 127) & ~(size_t)127;
+        size_t off = 128 + NST * stage;
+        const size_t ext_off = off;
+        if (any_ext) off += (size_t)2 * C * 2 * 32 * 16;
+        const size_t hist_off = off;
+        if (any_hist) off += (size_t)SPCG_CHAIN_HIST * 32 * 8;
+        const size_t warp = (off + 127) & ~(size_t)127;
+        if (warp * per_cta <= limit) {
+            D.C = C;
+            D.nst = NST;
+            D.stage_bytes = (uint32_t)stage;
+            D.warp_bytes = (uint32_t)warp;
+            D.ext_off = (uint32_t)ext_off;
+            D.hist_off = (uint32_t)hist_off;
+            D.any_ext = any_ext;
+            D.any_hist = any_hist;
+            *total = warp * per_cta;
+            return true;
+        }
+    }
+    return false;
+}
+
 spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay, int64_t n,
-                              bool identity_precond, spcg_device_t** out, int64_t* bytes) {
+                              bool identity_precond, const DevAllocator& alc, spcg_device_t** out,
+                              int64_t* bytes) {
     *out = nullptr;
     CK(cudaSetDevice(device));
     spcg_device_t* d = new spcg_device_t();
@@ -1571,14 +1633,42 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
     d->stream = (cudaStream_t)stream;
     d->strategy = lay.strategy;
     d->parts = lay.parts;
+    d->A = alc;
     Params& P = d->P;
     P.n = n;
     P.ring = lay.ring;
     P.identity = identity_precond ? 1 : 0;
-    P.A.nslices = lay.A.nslices;
-    UP(lay.A.eoff, P.A.eoff);
-    UP(lay.A.col, P.A.col);
-    UP(lay.A.val, P.A.val);
+    const bool wchain = lay.strategy == ST_WCHAIN;
+    const spcg::SpmvLayout& AL = wchain ? lay.C.A : lay.A;
+    // vectors of Algorithm 1: natural order, or execution (position) order for WCHAIN
+    const int64_t nv = wchain ? 32 * lay.C.nsteps : n;
+    d->mb_bytes = (size_t)nv * 16;
+    P.A.nslices = AL.nslices;
+    UP(AL.eoff, P.A.eoff);
+    UP(AL.col, P.A.col);
+    UP(AL.val, P.A.val);
+    if (wchain) {
+        const spcg::ChainLayout& CL = lay.C;
+        DevChain& D = P.CH;
+        D.nchains = CL.nchains;
+        D.per_cta = (CL.nchains + lay.parts - 1) / lay.parts;
+        D.W_L = CL.W_L;
+        D.W_U = CL.W_U;
+        D.rec_L = CL.rec_L;
+        D.rec_U = CL.rec_U;
+        D.nsteps = CL.nsteps;
+        D.npos = nv;
+        if (D.per_cta > NWARP || !chain_smem_config(CL, D.per_cta, D, &d->smem)) {
+            spcg::set_error("warp-chain layout: too many chains per CTA for shared memory");
+            spcg_dev_destroy(d);
+            return SPCG_ERR_INVALID_ARG;
+        }
+        UP(CL.chain_step, D.chain_step);
+        UP(CL.chain_flags, D.chain_flags);
+        UP(CL.recL, D.recL);
+        UP(CL.recU, D.recU);
+        UP(CL.perm, D.perm);
+    }
     if (upload_tri(d, lay.L, P.L) || upload_tri(d, lay.U, P.U)) { spcg_dev_destroy(d); return SPCG_ERR_CUDA; }
     UP(lay.part_begin, P.part_begin);
     UP(lay.S.bytes, P.stream);
@@ -1586,7 +1676,7 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
     UP(lay.S.part_uchunk, P.part_uchunk);
     UP(lay.S.chunk_bytes, P.chunk_bytes);
     void* p;
-    const size_t vb = (size_t)n * sizeof(double);
+    const size_t vb = (size_t)nv * sizeof(double);
 #define AL(bytes_, dst, T)                                                  \
     do {                                                                    \
         if (alloc(d, bytes_, &p)) { spcg_dev_destroy(d); return SPCG_ERR_OOM; } \
@@ -1597,24 +1687,31 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
     AL(vb, P.p, double*);
     AL(vb, P.z, double*);
     AL(vb, P.y, double*);
-    AL((size_t)n * 16, P.mbL, uint4*);
-    AL((size_t)n * 16, P.mbU, uint4*);
+    if (wchain) {
+        AL(vb, P.CH.xp, double*);
+        AL(vb, P.CH.bp, double*);
+        AL(vb, P.CH.t1, double*);
+    }
+    AL(d->mb_bytes, P.mbL, uint4*);
+    AL(d->mb_bytes, P.mbU, uint4*);
     AL(sizeof(double) * 3 * (size_t)lay.parts, P.partials, double*);
     AL(sizeof(Scal), P.sc, Scal*);
 #undef AL
-    if (cudaMemsetAsync(P.mbL, 0xFF, (size_t)n * 16, d->stream) != cudaSuccess ||
-        cudaMemsetAsync(P.mbU, 0xFF, (size_t)n * 16, d->stream) != cudaSuccess ||
+    if (cudaMemsetAsync(P.mbL, 0xFF, d->mb_bytes, d->stream) != cudaSuccess ||
+        cudaMemsetAsync(P.mbU, 0xFF, d->mb_bytes, d->stream) != cudaSuccess ||
         cudaMemsetAsync(P.sc, 0, sizeof(Scal), d->stream) != cudaSuccess) {
         spcg_dev_destroy(d);
         return SPCG_ERR_CUDA;
     }
-    d->smem = lay.strategy == ST_CHUNKED    ? chunked_smem_bytes(lay.ring)
-              : lay.strategy == ST_RESIDENT ? resident_smem_bytes(n)
-                                            : 0;
+    if (!wchain)
+        d->smem = lay.strategy == ST_CHUNKED    ? chunked_smem_bytes(lay.ring)
+                  : lay.strategy == ST_RESIDENT ? resident_smem_bytes(n)
+                                                : 0;
     void* kfn = pick_kernel(d->strategy);
     // one attribute value for every handle: the largest ring (or resident system) any layout builds
     const int smem_max = lay.strategy == ST_CHUNKED    ? (int)chunked_smem_bytes(SPCG_RING_MAX)
                          : lay.strategy == ST_RESIDENT ? (int)resident_smem_bytes(SPCG_RESIDENT_MAX_N)
+                         : wchain                      ? 227 * 1024 - 2048
                                                        : 0;
     if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max) != cudaSuccess) {
         spcg::set_error("cannot reserve shared memory for the ring");
@@ -1660,10 +1757,12 @@ void spcg_dev_destroy(spcg_device_t* d) {
     if (!d) return;
     cudaSetDevice(d->device);
     cudaStreamSynchronize(d->stream);
-    if (d->hist) cudaFree(d->hist);
-    if (d->stage) cudaFree(d->stage);
     if (d->sc_host) cudaFreeHost(d->sc_host);
-    for (void* p : d->allocs) cudaFree(p);
+    for (auto& a : d->allocs) {
+        if (d->A.free) d->A.free(a.first, a.second, (void*)d->stream, d->A.ctx);
+        else cudaFree(a.first);
+    }
+    d->allocs.clear();
     if (d->ev0) cudaEventDestroy(d->ev0);
     if (d->ev_bind) cudaEventDestroy(d->ev_bind);
     if (d->ev1) cudaEventDestroy(d->ev1);
@@ -1688,8 +1787,8 @@ static void report_abort(spcg_device_t* d, const Scal& sc) {
 // never carry a current epoch.
 static spcg_status_t reserve_epochs(spcg_device_t* d, unsigned long long need) {
     if ((unsigned long long)d->epoch + need < 0xFFFFFF00ull) return SPCG_OK;
-    CK(cudaMemsetAsync(d->P.mbL, 0xFF, (size_t)d->P.n * 16, d->stream));
-    CK(cudaMemsetAsync(d->P.mbU, 0xFF, (size_t)d->P.n * 16, d->stream));
+    CK(cudaMemsetAsync(d->P.mbL, 0xFF, d->mb_bytes, d->stream));
+    CK(cudaMemsetAsync(d->P.mbU, 0xFF, d->mb_bytes, d->stream));
     d->epoch = 1;
     return SPCG_OK;
 }
@@ -1726,9 +1825,12 @@ spcg_status_t spcg_dev_solve_begin(spcg_device_t* d, const double* b, double* x,
     d->epoch += (unsigned)(kmax + 3);
     long long cap = std::min<long long>(kmax + 1, 1 << 20);
     if (cap > d->hist_cap) {                 // persistent: no allocation on the solve path
-        if (d->hist) { CK(cudaStreamSynchronize(d->stream)); CK(cudaFree(d->hist)); d->hist = nullptr; }
+        if (d->hist) { CK(cudaStreamSynchronize(d->stream)); dev_free(d, d->hist); d->hist = nullptr; }
         d->hist_cap = std::max<long long>(cap, 1024);
-        CK(cudaMalloc((void**)&d->hist, sizeof(double) * d->hist_cap));
+        void* hp = nullptr;
+        spcg_status_t hs = dev_malloc(d, sizeof(double) * d->hist_cap, &hp);
+        if (hs != SPCG_OK) return hs;
+        d->hist = (double*)hp;
     }
     double* dh = d->hist;
     P.rhist = dh;
@@ -1832,7 +1934,12 @@ spcg_status_t spcg_dev_apply(spcg_device_t* d, int op, const double* in, double*
 spcg_status_t spcg_dev_copy(spcg_device_t* d, void* dst, const void* src, size_t bytes, int kind) {
     CK(cudaSetDevice(d->device));
     if (kind == -1) {          // the handle's staging buffer for host b, x: [0, n) and [n, 2n)
-        if (!d->stage) CK(cudaMalloc((void**)&d->stage, 2 * sizeof(double) * (size_t)d->P.n));
+        if (!d->stage) {
+            void* sp = nullptr;
+            spcg_status_t ss = dev_malloc(d, 2 * sizeof(double) * (size_t)d->P.n, &sp);
+            if (ss != SPCG_OK) return ss;
+            d->stage = (double*)sp;
+        }
         *(double**)dst = d->stage;
         return SPCG_OK;
     }

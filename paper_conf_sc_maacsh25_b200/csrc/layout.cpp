@@ -59,7 +59,7 @@ void build_spmv_layout(const Csr& A, SpmvLayout& out) {
 
 // one factor -> TriLayout
 static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev, int64_t w,
-                      int strategy, const std::vector<int64_t>& pb, int32_t ring, TriLayout& T) {
+                      int strategy, const std::vector<int64_t>& pb, int32_t ring, double wide_min, TriLayout& T) {
     const int64_t n = M.n;
     const int parts = (int)pb.size() - 1;
     auto dep_begin = [&](int64_t i) { return upper ? M.rp[i] + 1 : M.rp[i]; };   // U: skip diagonal
@@ -103,9 +103,8 @@ static void build_tri(const Csr& M, bool upper, const std::vector<int32_t>& lev,
     {
         int64_t deps = 0;
         for (int64_t i = 0; i < n; ++i) deps += dep_end(i) - dep_begin(i);
-        // experiment knob: SPCG_WIDE_MIN overrides the threshold (mean dependencies per row)
-        const char* wm = getenv("SPCG_WIDE_MIN");
-        const double wmin = wm ? atof(wm) : (double)SPCG_WCAP;
+        // threshold on the mean dependencies per row (spcg_options_t.wide_min; 0 = SPCG_WCAP)
+        const double wmin = wide_min > 0.0 ? wide_min : (double)SPCG_WCAP;
         T.wide = (strategy == SPCG_SPTRSV_LEVEL || strategy == SPCG_SPTRSV_SYNCFREE) && n > 0 &&
                  (double)deps / (double)n > wmin;
         if (T.wide) {
@@ -522,7 +521,7 @@ static bool partition_tiles(const Factors& F, int P, Partition& out) {
 }
 
 // Inspector: build candidate partitions and keep the one the model says is fastest.
-static void partition_rows(const Factors& F, int P, Partition& out, std::string* chosen) {
+static void partition_rows(const Factors& F, int P, int force_part, Partition& out, std::string* chosen) {
     const int64_t n = F.L.n;
     // microseconds per record without / with cross-CTA terms, handoff latency: measured on
     // B200 (tools/diag.py timelines)
@@ -548,16 +547,18 @@ static void partition_rows(const Factors& F, int P, Partition& out, std::string*
         Partition p;
         if (partition_tiles(F, P, p)) cand.push_back({"tiles", std::move(p)});
     }
-    const char* force = getenv("SPCG_PART");
+    static const char* kinds[] = {"contiguous", "strided", "affinity", "components", "tiles"};
+    const char* force = (force_part >= 0 && force_part < 5) ? kinds[force_part] : nullptr;
     double best = 1e300;
     size_t bi = 0;
+    bool forced = false;
     for (size_t c = 0; c < cand.size(); ++c) {
         // the model underrates the affinity partition (its rows' dependencies often go
         // through flags instead of the ring): measured 11 % slower than predicted relative
         // to strided on poisson3d 102^3, so it carries a 15 % penalty
         const double t = model_solve_time(F, cand[c].second, T_REC, T_EXT, H) * (cand[c].first == "affinity" ? 1.15 : 1.0);
-        if (getenv("SPCG_PART_VERBOSE")) fprintf(stderr, "[spcg] partition %s: modelled forward solve %.1f us\n", cand[c].first.c_str(), t);
-        if (force ? cand[c].first == force : t < best) { best = force ? 0.0 : t; bi = c; }
+        if (force && cand[c].first == force) { bi = c; forced = true; }
+        if (!forced && t < best) { best = t; bi = c; }
     }
     out = std::move(cand[bi].second);
     if (chosen) *chosen = cand[bi].first;
@@ -768,14 +769,15 @@ static void build_chunk_stream(const Factors& F, const Partition& PT, int32_t ri
     S.chunk_bytes.resize(S.part_chunk[parts], 16);
 }
 
-void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, Layouts& out) {
+void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, double wide_min, int force_part,
+                       Layouts& out) {
     const int64_t n = F.L.n;
     out.strategy = strategy;
     out.parts = parts;
     out.part_begin.assign(parts + 1, 0);
     if (strategy == SPCG_SPTRSV_CHUNKED) {
         Partition PT;
-        partition_rows(F, parts, PT, &out.partition);
+        partition_rows(F, parts, force_part, PT, &out.partition);
         // ring size: enough for the longest intra-part dependency distance in part-local
         // row numbering (slot = lidx & (ring - 1)), not the part size — a small ring leaves
         // shared memory to the L1 carve-out (layered 4096^2 SPCG: 8192 -> 64 entries).
@@ -820,8 +822,8 @@ void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, 
     out.part_begin[parts] = n;
     out.ring = 0;
     const std::vector<int64_t> pb{0, n};
-    build_tri(F.L, false, F.levL, F.wL, strategy, pb, out.ring, out.L);
-    build_tri(F.U, true, F.levU, F.wU, strategy, pb, out.ring, out.U);
+    build_tri(F.L, false, F.levL, F.wL, strategy, pb, out.ring, wide_min, out.L);
+    build_tri(F.U, true, F.levU, F.wU, strategy, pb, out.ring, wide_min, out.U);
 }
 
 }  // namespace spcg

@@ -13,13 +13,20 @@ from parity_util import check_x_elementwise
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
-EXECUTORS = ["level", "syncfree", "chunked", "resident"]
+EXECUTORS = ["level", "syncfree", "chunked", "resident", "wchain"]
 
 
-def _fits(ex, A):
-    """The resident executor takes n <= RESIDENT_MAX_N (one CTA's shared memory)."""
+def _fits(ex, A, K=0):
+    """The resident executor takes n <= RESIDENT_MAX_N (one CTA's shared memory); the
+    warp-chain executor rows of <= 16 dependencies (not 27-point ILU(2))."""
     if ex == "resident" and A.n > lib.RESIDENT_MAX_N:
         pytest.skip("resident executor: n > RESIDENT_MAX_N")
+    if ex == "wchain":
+        try:
+            lib.SPCG(A, K=K, sptrsv="wchain", device=-1).close()
+        except lib.SpcgError as e:
+            assert e.status == lib.ERR_INVALID_ARG
+            pytest.skip("warp-chain executor does not apply")
 
 
 def _dev(a):
@@ -40,7 +47,7 @@ SMALL = [("poisson2d", (37, 29), 0), ("poisson3d", (13, 11, 9), 0), ("fem_q1", (
 @pytest.mark.parametrize("parts", [1, 7, 0])
 def test_operators_match_oracle(fam, params, K, ex, parts):
     A = gen.make(fam, *params)
-    _fits(ex, A)
+    _fits(ex, A, K)
     h = lib.SPCG(A, mode="alg2", K=K, sptrsv=ex, parts=parts)
     L, U, _ = oracle.setup(A, mode="alg2", K=K)
     rng = np.random.default_rng(5)
@@ -76,7 +83,7 @@ def test_operators_match_oracle(fam, params, K, ex, parts):
 @pytest.mark.parametrize("ex", EXECUTORS)
 def test_pcg_matches_oracle(fam, params, K, mode, ex):
     A = gen.make(fam, *params)
-    _fits(ex, A)
+    _fits(ex, A, K)
     b, xt = gen.rhs(A)
     h = lib.SPCG(A, mode=mode, K=K, sptrsv=ex)
     L, U, _ = oracle.setup(A, mode=mode, K=K)

@@ -2,7 +2,8 @@
 emits, parsed independently here and checked against the factors the library
 exports (themselves bit-exact against the oracle in test_setup_parity.py).
 
-For every partition candidate (forced with SPCG_PART) and each section (L, U):
+For every partition candidate (forced with spcg_options_t.chunk_partition) and each
+section (L, U):
   * every row of the part appears in exactly one FIRST record, every row of the
     matrix in exactly one part;
   * rows come in non-decreasing wavefront level inside a part (the wavefront
@@ -54,10 +55,10 @@ CASES = [("poisson3d", (16, 16, 16), 0, 8), ("poisson3d", (13, 11, 9), 0, 7), ("
 
 @pytest.mark.parametrize("fam,params,K,parts", CASES)
 @pytest.mark.parametrize("part", ["contiguous", "strided", "affinity", "components", "tiles"])
-def test_record_stream_covers_factors(fam, params, K, parts, part, monkeypatch):
+def test_record_stream_covers_factors(fam, params, K, parts, part):
     A = gen.make(fam, *params)
-    monkeypatch.setenv("SPCG_PART", part)
-    h = lib.SPCG(A, mode="alg2", K=K, sptrsv="chunked", parts=parts, device=-1)
+    idx = ["contiguous", "strided", "affinity", "components", "tiles"].index(part)
+    h = lib.SPCG(A, mode="alg2", K=K, sptrsv="chunked", parts=parts, device=-1, chunk_partition=idx)
     if h.info["partition_name"] != part:
         pytest.skip(f"{part} is not a candidate for {fam}{params}")
     stream = h.export("dbg_stream")
