@@ -175,10 +175,30 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         // shuffle; otherwise the round-1 choice below.
         std::string chain_why;
         bool chain_built = false;
+        const int slots = sms * spcg_dev_ctas_per_sm();        // co-resident persistent CTAs
+        int chain_ctas = 0;
         if ((strategy == SPCG_SPTRSV_AUTO || strategy == SPCG_SPTRSV_WCHAIN) && !h->identity) {
             // components are packed onto as many chains as there are SMs (or the CTAs asked for)
-            const int target = opt.parts > 0 ? opt.parts : (opt.device >= 0 ? spcg_dev_sm_count(opt.device) : 148);
+            const int target = opt.parts > 0 ? opt.parts : sms;
             chain_built = build_chain_layout(h->A, h->F, std::max(1, target), h->lay.C, &chain_why);
+            if (chain_built) {
+                // CTAs: one per chain up to the SM count (more chains share CTAs, one solver
+                // warp each); large systems take every SM so the SpMV and vector phases use
+                // them all.  The chains of a CTA must fit its shared memory.
+                const int nch = h->lay.C.nchains;
+                const int64_t npos = 32 * h->lay.C.nsteps;
+                int p = opt.parts > 0 ? opt.parts : ((nch >= slots || npos >= (1 << 17)) ? slots : nch);
+                p = std::max(1, std::min<int>(p, slots));
+                if ((nch + p - 1) / p > 8) p = std::min(slots, (nch + 7) / 8);
+                ChainSmemCfg cfg;
+                if ((nch + p - 1) / p > 8 || !chain_smem_config(h->lay.C, (nch + p - 1) / p, cfg)) {
+                    chain_built = false;
+                    chain_why = "the chains per CTA do not fit shared memory";
+                    h->lay.C = ChainLayout();
+                } else {
+                    chain_ctas = p;
+                }
+            }
             if (chain_built) strategy = SPCG_SPTRSV_WCHAIN;
             else if (strategy == SPCG_SPTRSV_WCHAIN) {
                 delete h;
@@ -203,7 +223,6 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             set_error("the resident executor holds every vector in one CTA's shared memory: n <= SPCG_RESIDENT_MAX_N");
             return SPCG_ERR_INVALID_ARG;
         }
-        const int slots = sms * spcg_dev_ctas_per_sm();        // co-resident persistent CTAs
         int parts = opt.parts;
         // small systems: one CTA, except sync-free (wide ILU(K) rows), whose rows of a
         // wavefront spread over every warp of the grid (FEM 20^3 ILU(2), per iteration:
@@ -219,20 +238,7 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         }
         if (strategy == SPCG_SPTRSV_RESIDENT) parts = 1;
         if (strategy == SPCG_SPTRSV_WCHAIN) {
-            // CTAs: one per chain up to the SM count (more chains share CTAs, one solver warp
-            // each); large systems take every SM so the SpMV and vector phases use them all
-            const int nch = h->lay.C.nchains;
-            const int64_t npos = 32 * h->lay.C.nsteps;
-            if (opt.parts <= 0) parts = (nch >= slots || npos >= (1 << 17)) ? slots : nch;
-            parts = std::max(1, std::min<int>(parts, slots));
-            if ((nch + parts - 1) / parts > 8) {
-                parts = std::min(slots, (nch + 7) / 8);
-                if ((nch + parts - 1) / parts > 8) {
-                    delete h;
-                    set_error("warp-chain executor: more than 8 chains per CTA");
-                    return SPCG_ERR_INVALID_ARG;
-                }
-            }
+            parts = chain_ctas;
         } else {
             parts = std::max(1, std::min<int>(parts, slots));
             if ((int64_t)parts > h->n) parts = (int)h->n;

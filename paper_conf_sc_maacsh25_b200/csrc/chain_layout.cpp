@@ -265,8 +265,9 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
         out.iperm[i] = (int32_t)p;
     }
     out.partition = CP.name;
-    out.W_L = (int32_t)std::max<int64_t>(wl, 1);
-    out.W_U = (int32_t)std::max<int64_t>(wu, 1);
+    auto pow2 = [](int64_t w) { int64_t p = 1; while (p < w) p <<= 1; return (int32_t)p; };
+    out.W_L = pow2(std::max<int64_t>(wl, 1));
+    out.W_U = pow2(std::max<int64_t>(wu, 1));
     out.rec_L = 384 * out.W_L + 16;
     out.rec_U = 384 * out.W_U + 256 + 16;
     out.recL.assign((size_t)g * out.rec_L, 0);
@@ -280,7 +281,6 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
         const int rb = upper ? out.rec_U : out.rec_L;
         std::vector<uint8_t>& R = upper ? out.recU : out.recL;
         const size_t trailer = (size_t)384 * W + (upper ? 256 : 0);
-        std::vector<int32_t> next_ext(npos / 32 * 32 > 0 ? 0 : 0);
         for (int32_t c = 0; c < nch; ++c) {
             const int64_t s0 = out.chain_step[c], s1 = out.chain_step[c + 1];
             for (int64_t s = s0; s < s1; ++s) {
@@ -314,6 +314,7 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
                             } else {
                                 tag = ((uint32_t)CT_GLOB << 29) | (uint32_t)pj;
                                 flags |= CS_SLOW;
+                                out.chain_flags[c] |= upper ? CC_UGLOB : CC_LGLOB;
                                 out.glob_entries++;
                             }
                         } else {
@@ -325,6 +326,7 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
                             }
                             flags |= CS_SLOW | CS_EXT;
                             out.chain_flags[c] |= upper ? CC_UEXT : CC_LEXT;
+                            out.chain_flags[cj] |= upper ? CC_UPUB : CC_LPUB;
                             out.ext_entries++;
                             // the producer publishes its value with a ready flag
                             const int64_t sj = pj / 32;
@@ -334,8 +336,8 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
                             m |= 1u << (pj & 31);
                             std::memcpy(R.data() + pb, &m, 4);
                         }
-                        put<uint32_t>(R, base + (size_t)128 * k + 4 * l, tag);
-                        put<double>(R, base + (size_t)128 * W + (size_t)256 * k + 8 * l, M.val[q]);
+                        put<uint32_t>(R, base + 4 * ((size_t)W * l + k), tag);
+                        put<double>(R, base + (size_t)128 * W + 8 * ((size_t)W * l + k), M.val[q]);
                     }
                     if (upper) put<double>(R, base + (size_t)384 * W + 8 * l, 1.0 / M.val[M.rp[i]]);
                 }
@@ -348,17 +350,16 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
 
     // SpMV: SELL-32 of the ORIGINAL A over positions, one slice per step;
     // columns are positions, entries of a row in CSR order
+    // One width WA (the longest row of A) for every slice: slice s starts at entry column
+    // s * WA, so a warp streams any range of slices with two bulk copies and needs no
+    // offsets (stencil rows differ only at the boundary: little padding).
     SpmvLayout& S = out.A;
     S.nslices = (int32_t)g;
+    int64_t WA = 1;
+    for (int64_t i = 0; i < n; ++i) WA = std::max<int64_t>(WA, A.rp[i + 1] - A.rp[i]);
+    out.WA = (int32_t)WA;
     S.eoff.assign(g + 1, 0);
-    for (int64_t s = 0; s < g; ++s) {
-        int64_t w = 0;
-        for (int l = 0; l < 32; ++l) {
-            const int32_t i = out.perm[32 * s + l];
-            if (i >= 0) w = std::max<int64_t>(w, A.rp[i + 1] - A.rp[i]);
-        }
-        S.eoff[s + 1] = S.eoff[s] + w;
-    }
+    for (int64_t s = 0; s < g; ++s) S.eoff[s + 1] = S.eoff[s] + WA;
     S.col.assign(S.eoff[g] * 32, 0);
     S.val.assign(S.eoff[g] * 32, 0.0);
     for (int64_t s = 0; s < g; ++s)
@@ -377,6 +378,44 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
             }
         }
     return true;
+}
+
+}  // namespace spcg
+
+namespace spcg {
+
+bool chain_smem_config(const ChainLayout& CL, int per_cta, ChainSmemCfg& out) {
+    const size_t C = SPCG_CHAIN_C;
+    const size_t step_bytes = std::max<size_t>((size_t)CL.rec_L + 4 * 256, (size_t)CL.rec_U + 2 * 256);
+    const bool any_ext = CL.ext_entries > 0, any_hist = CL.hist_entries > 0;
+    const size_t limit = SPCG_CHAIN_SMEM_LIMIT;
+    const size_t stage = (C * step_bytes + 127) & ~(size_t)127;
+    for (int NST = 16; NST >= 2; --NST) {
+        size_t off = NST * stage;
+        const size_t ext_off = off;
+        if (any_ext) off += 2 * C * 2 * 32 * 16;
+        const size_t hist_off = off;
+        if (any_hist) off += (size_t)SPCG_CHAIN_HIST * 32 * 8;
+        const size_t warp = (off + 127) & ~(size_t)127;
+        if (warp * per_cta <= limit) {
+            out.nst = NST;
+            out.stage_bytes = (uint32_t)stage;
+            out.warp_bytes = (uint32_t)warp;
+            out.ext_off = (uint32_t)ext_off;
+            out.hist_off = (uint32_t)hist_off;
+            out.cta_bytes = warp * per_cta;
+            // SpMV staging (the same shared memory, used between the triangular solves):
+            // 8 warps x sp_nst stages of SPCG_SPMV_G slices of WA entry columns
+            const size_t sp_stage = (size_t)SPCG_SPMV_G * CL.WA * 384;
+            out.sp_nst = 0;
+            out.sp_stage_bytes = (uint32_t)sp_stage;
+            for (int sn = 3; sn >= 2; --sn)
+                if (8 * sn * sp_stage <= limit) { out.sp_nst = sn; break; }
+            out.cta_bytes = std::max(out.cta_bytes, 8 * (size_t)out.sp_nst * sp_stage);
+            return true;
+        }
+    }
+    return false;
 }
 
 }  // namespace spcg

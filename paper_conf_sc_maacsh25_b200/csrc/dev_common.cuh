@@ -69,10 +69,12 @@ struct Scal {
 // warp-chain executor (wchain.cu; layout: chain_layout.cpp, internal.h ChainLayout)
 struct DevChain {
     int32_t nchains, per_cta;      // chains, solver warps per CTA (chain c -> CTA c % grid, warp c / grid)
-    int32_t C, nst;                // steps per stage (chunk), stages per solver warp
+    int32_t nst;                   // stages per solver warp (SPCG_CHAIN_C steps each)
     int32_t W_L, W_U, rec_L, rec_U;
     int32_t any_ext, any_hist;
     uint32_t stage_bytes, warp_bytes, ext_off, hist_off;
+    int32_t WA, sp_nst;            // SpMV: uniform slice width, TMA stages per warp (0: register path)
+    uint32_t sp_stage_bytes;
     int64_t nsteps, npos;
     const int64_t* chain_step;     // [nchains+1]
     const uint32_t* chain_flags;   // [nchains] CC_*
@@ -352,12 +354,15 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* b) {
 __device__ __forceinline__ void mbar_arrive_tx(uint64_t* b, unsigned bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
 }
+#ifndef SPCG_MBAR_SUSPEND_NS
+#define SPCG_MBAR_SUSPEND_NS 20000   // try_wait suspend-time hint (ns): the warp sleeps until the phase completes
+#endif
 __device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
     unsigned ok;
     asm volatile(
         "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\tselp.u32 %0, 1, 0, p;\n\t}"
         : "=r"(ok)
-        : "r"(smem_u32(b)), "r"(parity), "r"(20000u)   // suspend (HW sleep) until the phase completes (<= 20 us)
+        : "r"(smem_u32(b)), "r"(parity), "r"((unsigned)SPCG_MBAR_SUSPEND_NS)   // HW sleep until the phase completes
         : "memory");
     return ok != 0;
 }

@@ -137,20 +137,23 @@ struct ChunkStream {
 // order of L is one of U, the ILU(K) pattern being symmetric).  All vectors of
 // Algorithm 1 live in execution ("position") order pos = 32 * global_step + lane for
 // the whole solve; b and x are permuted on entry and exit.  A record per step holds,
-// per lane, W dependency tags + values (and 1/u_ii for U):
-//   tag u32: kind << 29 | payload
-//     PAD  (0): no entry (value 0)
-//     PREV (1): the value lane `payload & 31` produced in the chain's previous step
-//               (a warp shuffle, no memory access)
-//     HIST (2): lane payload & 31, `(payload >> 5) & 255` steps back (shared-memory ring)
-//     GLOB (3): own chain, older than the ring: position payload, read from global
-//     EXT  (4): another chain: position payload & (2^28-1), ordinal (payload >> 28) & 1
+// lane-major, W (a power of two) dependency tags + values (and 1/u_ii for U):
+//   tag u32 [32][W] at 0, value f64 [32][W] at 128 W, (U) 1/u_ii f64 [32] at 384 W,
+//   trailer {u32 publish mask (lanes whose value another chain reads), u32 flags}.
+//   tag = kind << 29 | payload:
+//     PREV (0): payload = the lane whose previous-step value is the dependency (a warp
+//               shuffle, no memory access); padding entries are PREV lane 0, value 0
+//     HIST (1): lane payload & 31, `(payload >> 5) & 255` steps back (shared-memory ring)
+//     GLOB (2): own chain, older than the ring: position payload, read from global
+//     EXT  (3): another chain: position payload & (2^28-1), ordinal (payload >> 28) & 1
 //               of the lane's prefetched flags (ready flag prefetched one chunk ahead)
-//     EXTS (5): another chain, beyond two per lane and step: polled at use
-//   trailer: u32 publish mask (lanes whose value another chain reads), u32 flags.
-enum { CT_PAD = 0, CT_PREV = 1, CT_HIST = 2, CT_GLOB = 3, CT_EXT = 4, CT_EXTS = 5 };
+//     EXTS (4): another chain, beyond two per lane and step: polled at use
+enum { CT_PREV = 0, CT_HIST = 1, CT_GLOB = 2, CT_EXT = 3, CT_EXTS = 4 };
 enum { CS_SLOW = 1, CS_EXT = 2 };                 // record trailer flags
-enum { CC_LHIST = 1, CC_LEXT = 2, CC_UHIST = 4, CC_UEXT = 8 };   // per-chain flags
+// per-chain flags: which kinds a pass of the chain uses (the kernel picks the plain
+// shuffle-only step body when none is set)
+enum { CC_LHIST = 1, CC_LEXT = 2, CC_UHIST = 4, CC_UEXT = 8, CC_LGLOB = 16, CC_UGLOB = 32, CC_LPUB = 64,
+       CC_UPUB = 128 };
 constexpr int SPCG_CHAIN_WMAX = 16;              // dependency columns per record (wider: other executors)
 constexpr int SPCG_CHAIN_HIST = 32;              // steps kept in the per-warp history ring
 
@@ -164,13 +167,30 @@ struct ChainLayout {
     std::vector<int32_t> perm;            // [npos] row at each position (-1 padding)
     std::vector<int32_t> iperm;           // [n] position of each row
     std::vector<uint8_t> recL, recU;      // nsteps records each
-    SpmvLayout A;                         // SELL-32 of A over positions (slice = step)
+    SpmvLayout A;                         // SELL-32 of A over positions (slice = step), uniform width WA
+    int32_t WA = 0;
     std::string partition;                // components / grid2d / grid3d
     int64_t ext_entries = 0, hist_entries = 0, glob_entries = 0, prev_entries = 0;
 };
 // Builds the chain layout when the factors suit it (dependency columns <= WMAX, a
 // partition into chains found); returns false (why set) otherwise.
 bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, ChainLayout& out, std::string* why);
+
+// Shared memory of the warp-chain kernel per solver warp: mbarriers (128 B), NST stages
+// of SPCG_CHAIN_C steps (records + the pass's operand slices), the prefetched-flag queue,
+// the history ring.  The most stages (2..16) whose per-CTA total fits; false if none.
+constexpr int SPCG_CHAIN_C = 8;                  // steps per stage (compile-time in the kernel)
+struct ChainSmemCfg {
+    int32_t nst = 0;
+    uint32_t stage_bytes = 0, warp_bytes = 0, ext_off = 0, hist_off = 0;
+    int32_t sp_nst = 0;                   // SpMV: stages per warp (0: register path), SPCG_SPMV_G slices each
+    uint32_t sp_stage_bytes = 0;
+    size_t cta_bytes = 0;                 // max of the triangular-solve and SpMV needs
+};
+constexpr int SPCG_SPMV_G = 4;           // SpMV slices per TMA stage
+// dynamic shared memory of the warp-chain kernel: 227 KB per CTA minus its static blocks
+constexpr size_t SPCG_CHAIN_SMEM_LIMIT = 227 * 1024 - 4096;
+bool chain_smem_config(const ChainLayout& CL, int per_cta, ChainSmemCfg& out);
 
 struct Layouts {
     int32_t strategy = SPCG_SPTRSV_LEVEL;

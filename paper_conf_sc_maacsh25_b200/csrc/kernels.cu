@@ -1590,39 +1590,6 @@ static void* pick_kernel(int strategy) {
     }
 }
 
-// WCHAIN shared memory per solver warp: mbarriers, NST stages of C steps (records + the
-// pass's operand slices), the prefetched-flag queue, the history ring.  The largest
-// (C, NST) whose per-CTA total fits.
-static bool chain_smem_config(const spcg::ChainLayout& CL, int per_cta, DevChain& D, size_t* total) {
-    const size_t step_bytes = std::max<size_t>((size_t)CL.rec_L + 4 * 256, (size_t)CL.rec_U + 2 * 256);
-    const bool any_ext = CL.ext_entries > 0, any_hist = CL.hist_entries > 0;
-    static const int cfg[][2] = {{8, 4}, {8, 3}, {4, 4}, {4, 3}, {4, 2}, {2, 2}, {1, 2}};
-    const size_t limit = 227 * 1024 - 2048;       // dynamic smem per CTA, minus the static blocks
-    for (auto& cn : cfg) {
-        const int C = cn[0], NST = cn[1];
-        const size_t stage = (C * step_bytes + 127) & ~(size_t)127;
-        size_t off = 128 + NST * stage;
-        const size_t ext_off = off;
-        if (any_ext) off += (size_t)2 * C * 2 * 32 * 16;
-        const size_t hist_off = off;
-        if (any_hist) off += (size_t)SPCG_CHAIN_HIST * 32 * 8;
-        const size_t warp = (off + 127) & ~(size_t)127;
-        if (warp * per_cta <= limit) {
-            D.C = C;
-            D.nst = NST;
-            D.stage_bytes = (uint32_t)stage;
-            D.warp_bytes = (uint32_t)warp;
-            D.ext_off = (uint32_t)ext_off;
-            D.hist_off = (uint32_t)hist_off;
-            D.any_ext = any_ext;
-            D.any_hist = any_hist;
-            *total = warp * per_cta;
-            return true;
-        }
-    }
-    return false;
-}
-
 spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay, int64_t n,
                               bool identity_precond, const DevAllocator& alc, spcg_device_t** out,
                               int64_t* bytes) {
@@ -1658,11 +1625,23 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         D.rec_U = CL.rec_U;
         D.nsteps = CL.nsteps;
         D.npos = nv;
-        if (D.per_cta > NWARP || !chain_smem_config(CL, D.per_cta, D, &d->smem)) {
+        spcg::ChainSmemCfg cfg;
+        if (D.per_cta > NWARP || !spcg::chain_smem_config(CL, D.per_cta, cfg)) {
             spcg::set_error("warp-chain layout: too many chains per CTA for shared memory");
             spcg_dev_destroy(d);
             return SPCG_ERR_INVALID_ARG;
         }
+        D.nst = cfg.nst;
+        D.stage_bytes = cfg.stage_bytes;
+        D.warp_bytes = cfg.warp_bytes;
+        D.ext_off = cfg.ext_off;
+        D.hist_off = cfg.hist_off;
+        D.WA = CL.WA;
+        D.sp_nst = cfg.sp_nst;
+        D.sp_stage_bytes = cfg.sp_stage_bytes;
+        D.any_ext = CL.ext_entries > 0;
+        D.any_hist = CL.hist_entries > 0;
+        d->smem = cfg.cta_bytes;
         UP(CL.chain_step, D.chain_step);
         UP(CL.chain_flags, D.chain_flags);
         UP(CL.recL, D.recL);
@@ -1711,7 +1690,7 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
     // one attribute value for every handle: the largest ring (or resident system) any layout builds
     const int smem_max = lay.strategy == ST_CHUNKED    ? (int)chunked_smem_bytes(SPCG_RING_MAX)
                          : lay.strategy == ST_RESIDENT ? (int)resident_smem_bytes(SPCG_RESIDENT_MAX_N)
-                         : wchain                      ? 227 * 1024 - 2048
+                         : wchain                      ? (int)spcg::SPCG_CHAIN_SMEM_LIMIT
                                                        : 0;
     if (cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max) != cudaSuccess) {
         spcg::set_error("cannot reserve shared memory for the ring");

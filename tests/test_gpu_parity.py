@@ -16,14 +16,14 @@ pytestmark = pytest.mark.gpu
 EXECUTORS = ["level", "syncfree", "chunked", "resident", "wchain"]
 
 
-def _fits(ex, A, K=0):
+def _fits(ex, A, K=0, parts=0):
     """The resident executor takes n <= RESIDENT_MAX_N (one CTA's shared memory); the
     warp-chain executor rows of <= 16 dependencies (not 27-point ILU(2))."""
     if ex == "resident" and A.n > lib.RESIDENT_MAX_N:
         pytest.skip("resident executor: n > RESIDENT_MAX_N")
     if ex == "wchain":
         try:
-            lib.SPCG(A, K=K, sptrsv="wchain", device=-1).close()
+            lib.SPCG(A, K=K, sptrsv="wchain", parts=parts, device=-1).close()
         except lib.SpcgError as e:
             assert e.status == lib.ERR_INVALID_ARG
             pytest.skip("warp-chain executor does not apply")
@@ -47,7 +47,7 @@ SMALL = [("poisson2d", (37, 29), 0), ("poisson3d", (13, 11, 9), 0), ("fem_q1", (
 @pytest.mark.parametrize("parts", [1, 7, 0])
 def test_operators_match_oracle(fam, params, K, ex, parts):
     A = gen.make(fam, *params)
-    _fits(ex, A, K)
+    _fits(ex, A, K, parts)
     h = lib.SPCG(A, mode="alg2", K=K, sptrsv=ex, parts=parts)
     L, U, _ = oracle.setup(A, mode="alg2", K=K)
     rng = np.random.default_rng(5)
