@@ -343,6 +343,46 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
                     cpa16(qb + ((size_t)t * 2 + ((tg[k] >> 28) & 1)) * 32 + lane, mb + (tg[k] & 0x0fffffffu));
         }
     };
+    // Before a chunk runs, every prefetched flag that was still stale is polled again, all
+    // of them together, until current: the chain then waits at most once per chunk (not
+    // once per step), and the wait re-establishes a lag behind the producing chain of
+    // about a chunk, so later prefetches find their values ready.
+    auto settle_ext = [&](int q) {
+        int64_t glo;
+        int cnt;
+        chunk_range(q, glo, cnt);
+        const uint8_t* st = stage_of(q);
+        uint4* qb = WS.extq + (size_t)(q & 1) * CC * 64;
+        const long long t0 = clock64();
+        for (;;) {
+            bool stale = false;
+            for (int i = 0; i < cnt; ++i) {
+                const uint8_t* R = st + (size_t)i * RECB;
+                const int t = UPPER ? cnt - 1 - i : i;
+                uint32_t tg[W];
+                lds_tags<W>(R + 4 * W * lane, tg);
+#pragma unroll
+                for (int k = 0; k < W; ++k)
+                    if ((tg[k] >> 29) == CT_EXT) {
+                        uint4* slot = qb + ((size_t)t * 2 + ((tg[k] >> 28) & 1)) * 32 + lane;
+                        uint4 f = *slot;
+                        if (f.y != ep || f.w != ep) {
+                            asm volatile("ld.volatile.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                                         : "=r"(f.x), "=r"(f.y), "=r"(f.z), "=r"(f.w)
+                                         : "l"(mb + (tg[k] & 0x0fffffffu))
+                                         : "memory");
+                            *slot = f;
+                            if (f.y != ep || f.w != ep) stale = true;
+                        }
+                    }
+            }
+            if (!__any_sync(0xffffffffu, stale)) break;
+            if (__any_sync(0xffffffffu, ld_volatile_int(&E.sc->abort) != 0 || clock64() - t0 > SPIN_TIMEOUT_CYC)) {
+                if (lane == 0) atomicExch(&E.sc->abort, 1);
+                break;
+            }
+        }
+    };
     const bool refill = ROLE == 0 || (ROLE == 1) == !UPPER;   // the last reader of a stage refills it
 
     long long t_pass = SPCG_CHAIN_PROF ? clock64() : 0, t_wait = 0, t_ext = 0;
@@ -382,6 +422,7 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
             cpa_commit();
             cpa_wait1();                                    // chunk q's flags landed
             G.qb = WS.extq + (size_t)(q & 1) * CC * 64;
+            if (use_ext) settle_ext(q);
         }
         if (SPCG_CHAIN_PROF) { t_ext += clock64() - t0; t0 = clock64(); }
         if (!wait_bar(SPLIT && !UPPER ? WS.hand : WS.full, q)) return;
@@ -606,11 +647,14 @@ __device__ void chain_spmv_tma(const DevChain& D, const DevA& A, uint8_t* dyn, u
         bulk_g2s(st, A.col + s * WA * 32, cb, &bar[slot]);
         bulk_g2s(st + (size_t)G * WA * 128, A.val + s * WA * 32, vb, &bar[slot]);
     };
+    long long t_all = SPCG_CHAIN_PROF ? clock64() : 0, t_wait = 0;
     if (lane == 0)
         for (int j = 0; j < min(NS, nst); ++j) issue(j);
     for (int j = 0; j < nst; ++j) {
         const unsigned u = spq + j;
+        const long long tw = SPCG_CHAIN_PROF ? clock64() : 0;
         if (!warp_ok(mbar_wait(&bar[u % NS], (u / NS) & 1, sc))) return;
+        if (SPCG_CHAIN_PROF) t_wait += clock64() - tw;
         const uint8_t* st = ring + (size_t)(u % NS) * D.sp_stage_bytes;
         const int32_t* cs = (const int32_t*)st;
         const double* vs = (const double*)(st + (size_t)G * WA * 128);
@@ -628,6 +672,10 @@ __device__ void chain_spmv_tma(const DevChain& D, const DevA& A, uint8_t* dyn, u
         if (lane == 0 && j + NS < nst) issue(j + NS);
     }
     spq += (unsigned)nst;
+    if (SPCG_CHAIN_PROF && lane == 0 && g_chain_prof) {
+        atomicAdd(g_chain_prof + 22, (unsigned long long)t_wait);
+        atomicAdd(g_chain_prof + 23, (unsigned long long)(clock64() - t_all));
+    }
 }
 
 // the SpMV of the iteration: TMA-streamed for uniform widths 3..8, the register path otherwise

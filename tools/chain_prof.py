@@ -54,7 +54,8 @@ def main():
                            gen_passes=v[o + 5])
         it = max(k, 1) * int(out["ctas"])
         out["phase_cyc_per_iter_per_cta"] = dict(spmv=v[16] / it, spmv_bar=v[17] / it, tri=v[18] / it,
-                                                 tri_bar=v[19] / it, pupd=v[20] / it, pupd_bar=v[21] / it)
+                                                 tri_bar=v[19] / it, pupd=v[20] / it, pupd_bar=v[21] / it,
+                                                 spmv_warp_wait=v[22] / it / 8, spmv_warp_total=v[23] / it / 8)
     print(json.dumps(out))
 
 
