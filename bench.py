@@ -215,6 +215,7 @@ def main():
     ap.add_argument("--sptrsv", default="auto")
     ap.add_argument("--parts", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-host-setup", action="store_true", help="skip timing the host setup beside the GPU one")
     ap.add_argument("--batch-count", type=int, default=64)
     ap.add_argument("--lanes", type=int, default=4,
                     help="C5: concurrent streams per GPU (each with SMs/lanes persistent CTAs)")
@@ -259,9 +260,19 @@ def main():
     torch.cuda.set_device(dev)
     stream = torch.cuda.current_stream(dev)
 
+    # NEXT-1: ILU(0) systems are set up on the GPU (validation, Algorithm 2, ILU(0), level
+    # sets: gsetup.cu); the host setup of the same products is timed once for comparison
+    setup_kind = "gpu" if K == 0 else "host"
     handles = {}
     for mode in ("alg2", "none"):
-        handles[mode] = spcg.SPCG(A, mode=mode, K=K, sptrsv=args.sptrsv, parts=args.parts, device=dev, stream=stream)
+        handles[mode] = spcg.SPCG(A, mode=mode, K=K, sptrsv=args.sptrsv, parts=args.parts, device=dev, stream=stream,
+                                  setup=setup_kind)
+    host_setup_ms = None
+    if K == 0 and not args.no_host_setup:
+        hh = spcg.SPCG(A, mode="alg2", K=K, sptrsv=args.sptrsv, parts=args.parts, device=dev, stream=stream,
+                       setup="host")
+        host_setup_ms = hh.info["setup_ms_total"]
+        hh.close()
     bd = torch.from_numpy(b).to(f"cuda:{dev}")
     xd = torch.empty_like(bd)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=f"cuda:{dev}")
@@ -310,7 +321,7 @@ def main():
     sweep = []
     for t in [float(v) for v in sweep_spec.split(",") if v.strip()]:
         hs = spcg.SPCG(A, mode="fixed", fixed_pct=t, K=K, sptrsv=args.sptrsv, parts=args.parts, device=dev,
-                       stream=stream)
+                       stream=stream, setup=setup_kind)
         hs.solve(bd, xd, EPS, KMAX)
         tms, tk = [], 0
         for _ in range(max(1, min(args.steps, 3))):
@@ -395,6 +406,14 @@ def main():
         "gpu_launches": args.steps,
         "clocks": clocks,
         "setup_ms": {k: si[k] for k in si if k.startswith("setup_ms")},
+        # NEXT-1 / §4.3: end to end = setup (on the GPU for ILU(0)) + iterative phase
+        "end_to_end": {
+            "setup": setup_kind,
+            "spcg_setup_ms": si["setup_ms_total"], "pcg_setup_ms": pi["setup_ms_total"],
+            "spcg_host_setup_ms": host_setup_ms,
+            "spcg_ms": si["setup_ms_total"] + s_ms, "pcg_ms": pi["setup_ms_total"] + p_ms,
+            "speedup_spcg_vs_pcg": (pi["setup_ms_total"] + p_ms) / (si["setup_ms_total"] + s_ms),
+            "paper_context": "1.68x (ILU(0)) / 3.73x (ILU(K)) end to end, A100 fp32 (P:L56-58)"},
     }
     print(json.dumps(line))
     if ws > 1:

@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define SPCG_ABI_VERSION 2
+#define SPCG_ABI_VERSION 3
 
 typedef int32_t spcg_status_t;
 enum {
@@ -111,6 +111,8 @@ enum {
                                    persistent kernel replaces); setup returns SPCG_ERR_INVALID_ARG */
 };
 
+enum { SPCG_SETUP_HOST = 0, SPCG_SETUP_GPU = 1 };
+
 /* Device allocator hooks: when dev_alloc is set, every device buffer the handle owns
  * comes from dev_alloc(bytes, stream, ctx) and goes back through
  * dev_free(ptr, bytes, stream, ctx) (e.g. PyTorch's caching allocator; the Python
@@ -135,7 +137,12 @@ typedef struct {
                                    row (0 = default SPCG_WCAP = 8) */
     int32_t chunk_partition;    /* CHUNKED executor: -1 = inspector's choice (default), else force
                                    0 contiguous, 1 strided, 2 affinity, 3 components, 4 tiles */
-    int32_t reserved[7];
+    int32_t setup_device;       /* SPCG_SETUP_HOST (default) or SPCG_SETUP_GPU: validation, Algorithm 2,
+                                   ILU(0) and the level sets on the GPU (NEXT-1; K = 0 only — K > 0 and
+                                   K = -1 run on the host).  Products are bit-exact with the host setup
+                                   except the Frobenius indicator values, which agree up to summation
+                                   order (reading A6g) */
+    int32_t reserved[6];
 } spcg_options_t;
 
 typedef struct {
@@ -165,6 +172,8 @@ typedef struct {
     int32_t chains;             /* WCHAIN: warp chains (0 otherwise) */
     int64_t positions;          /* WCHAIN: execution-order slots (32 x steps >= n) */
     int64_t chain_entries[4];   /* WCHAIN: dependencies read by shuffle / shared ring / global / flag */
+    int32_t setup_device;       /* where validation .. ILU ran: SPCG_SETUP_HOST / SPCG_SETUP_GPU */
+    double setup_ms_total;      /* spcg_setup wall time, entry to return */
 } spcg_setup_info_t;
 
 typedef struct {
@@ -279,6 +288,16 @@ typedef struct {
     double flag_relaxed_cross_die_ns;
 } spcg_calib_t;
 spcg_status_t spcg_calibrate(int32_t device, spcg_calib_t* out);
+
+/* Ready-flag stress test (robustness of the "LL" flags of the sync-free, chunked and
+ * warp-chain executors): a value is published as one 16-byte volatile
+ * store {lo32, epoch, hi32, epoch} and accepted when both epochs read current, which
+ * is sound only if each 8-byte half is observed whole.  Half of the SMs rewrite
+ * `nslots` slots `rounds` times (one epoch per round), the other half poll them at
+ * random throughout.  out[0] = torn reads (epochs agree, value halves from another
+ * epoch: must be 0), out[1] = reads whose epochs differ (benign), out[2] = good reads.
+ * Errors: SPCG_ERR_INVALID_ARG (out == NULL, sizes <= 0), SPCG_ERR_OOM, SPCG_ERR_CUDA. */
+spcg_status_t spcg_ll_stress(int32_t device, int32_t nslots, int32_t rounds, uint64_t* out);
 
 #ifdef __cplusplus
 }

@@ -77,7 +77,7 @@ class Options(ctypes.Structure):
                 ("parts", ctypes.c_int32), ("host_threads", ctypes.c_int32), ("exec", ctypes.c_int32),
                 ("dev_alloc", _ALLOC_FN), ("dev_free", _FREE_FN), ("alloc_ctx", ctypes.c_void_p),
                 ("wide_min", ctypes.c_double), ("chunk_partition", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 7)]
+                ("setup_device", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
 
 
 class SetupInfo(ctypes.Structure):
@@ -93,7 +93,8 @@ class SetupInfo(ctypes.Structure):
                 ("sptrsv", ctypes.c_int32), ("parts", ctypes.c_int32), ("device_bytes", ctypes.c_int64),
                 ("algo_bytes_per_iter", ctypes.c_double), ("algo_flops_per_iter", ctypes.c_double),
                 ("partition", ctypes.c_int32), ("chains", ctypes.c_int32), ("positions", ctypes.c_int64),
-                ("chain_entries", ctypes.c_int64 * 4)]
+                ("chain_entries", ctypes.c_int64 * 4), ("setup_device", ctypes.c_int32),
+                ("setup_ms_total", ctypes.c_double)]
 
 
 class SolveInfo(ctypes.Structure):
@@ -104,7 +105,7 @@ class SolveInfo(ctypes.Structure):
 EXPORTED = ["spcg_abi_version", "spcg_status_string", "spcg_last_error", "spcg_drop_params_default",
             "spcg_options_default", "spcg_setup", "spcg_get_setup_info", "spcg_solve", "spcg_apply_spmv",
             "spcg_apply_lower", "spcg_apply_upper", "spcg_apply_precond", "spcg_export", "spcg_destroy",
-            "spcg_calibrate", "spcg_solve_async", "spcg_solve_wait", "spcg_set_stream"]
+            "spcg_calibrate", "spcg_solve_async", "spcg_solve_wait", "spcg_set_stream", "spcg_ll_stress"]
 
 
 def load(path: str | None = None):
@@ -150,7 +151,9 @@ def load(path: str | None = None):
     lib.spcg_set_stream.restype = I32
     lib.spcg_calibrate.argtypes = [I32, ctypes.POINTER(Calib)]
     lib.spcg_calibrate.restype = I32
-    if lib.spcg_abi_version() != 2:
+    lib.spcg_ll_stress.argtypes = [I32, I32, I32, ctypes.POINTER(ctypes.c_uint64)]
+    lib.spcg_ll_stress.restype = I32
+    if lib.spcg_abi_version() != 3:
         raise ImportError("libspcg ABI version mismatch")
     _lib = lib
     return lib
@@ -169,6 +172,13 @@ def calibrate(device: int = 0) -> dict:
     c = Calib()
     _check(load().spcg_calibrate(device, ctypes.byref(c)), "spcg_calibrate")
     return {f: getattr(c, f) for f, _ in Calib._fields_}
+
+
+def ll_stress(device: int = 0, nslots: int = 4096, rounds: int = 2000) -> dict:
+    """spcg_ll_stress: torn / mixed / good reads of the 16-byte LL ready flags."""
+    out = (ctypes.c_uint64 * 3)()
+    _check(load().spcg_ll_stress(device, nslots, rounds, out), "spcg_ll_stress")
+    return {"torn": int(out[0]), "mixed": int(out[1]), "ok": int(out[2])}
 
 
 def _check(st, what=""):
@@ -233,10 +243,13 @@ class SPCG:
     """A set-up SPCG preconditioner + solver bound to one device (or host-only, device=-1).
 
     allocator: "torch" (default: device buffers from PyTorch's caching allocator through
-    the spcg_options_t hooks) or "cuda" (the library's own cudaMalloc)."""
+    the spcg_options_t hooks) or "cuda" (the library's own cudaMalloc).
+    setup: "host" (default) or "gpu" (NEXT-1: validation, Algorithm 2, ILU(0) and the
+    level sets on the device; K = 0 only, other K run on the host)."""
 
     def __init__(self, A, mode="alg2", K=0, fixed_pct=0.0, sptrsv="auto", parts=0, device=0, stream=None,
-                 host_threads=0, allocator="torch", exec="auto", wide_min=0.0, chunk_partition=-1, **drop_kw):
+                 host_threads=0, allocator="torch", exec="auto", wide_min=0.0, chunk_partition=-1, setup="host",
+                 **drop_kw):
         lib = load()
         rp = np.ascontiguousarray(A.row_ptr, np.int64)
         col = np.ascontiguousarray(A.col, np.int32)
@@ -253,6 +266,7 @@ class SPCG:
         opt.exec = EXEC[exec]
         opt.wide_min = wide_min
         opt.chunk_partition = chunk_partition
+        opt.setup_device = {"host": 0, "gpu": 1}[setup]
         self.device = device
         self._alloc = None
         if device >= 0:

@@ -34,31 +34,53 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     lib = out or LIB
     if not force and not defines and out is None and not stale():
         return LIB
+    import time
+    t_start = time.time()
     bdir = os.path.join(HERE, "build" if not defines else "build_" + "_".join(d.strip("-D").replace("=", "") for d in defines))
     os.makedirs(bdir, exist_ok=True)
-    objs = []
+    jobs = []
     for cu in sorted(glob.glob(os.path.join(CSRC, "*.cu"))):
         o = os.path.join(bdir, os.path.basename(cu) + ".o")
         cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
                "-I", os.path.join(ROOT, "include"), *defines, "-c", cu, "-o", o]
-        r = subprocess.run(cmd, capture_output=True, text=True)
-        if r.returncode != 0:
-            raise RuntimeError(f"nvcc failed:\n{r.stderr}")
-        if verbose:
-            print(r.stderr)
-        with open(os.path.join(bdir, "ptxas.log"), "w") as f:
-            f.write(r.stderr)
-        objs.append(o)
+        jobs.append((cu, o, cmd))
     for cpp in sorted(glob.glob(os.path.join(CSRC, "*.cpp"))):
         o = os.path.join(bdir, os.path.basename(cpp) + ".o")
         cmd = ["g++", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-fPIC", "-std=c++17",
                "-I", os.path.join(ROOT, "include"), "-I", "/usr/local/cuda/include", *defines, "-c", cpp, "-o", o]
-        subprocess.check_call(cmd)
+        jobs.append((cpp, o, cmd))
+    # translation units compile in parallel (wchain.cu alone takes minutes); an object newer
+    # than its source and every header is reused
+    hdrs = [h for h in _sources() if h.endswith((".h", ".cuh"))]
+    hdr_t = max(os.path.getmtime(h) for h in hdrs)
+
+    def fresh(src, o):
+        return not force and os.path.exists(o) and os.path.getmtime(o) >= max(os.path.getmtime(src), hdr_t)
+
+    procs = [(src, o, None if fresh(src, o) else
+              subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True))
+             for src, o, cmd in jobs]
+    objs, logs = [], []
+    for src, o, pr in procs:
         objs.append(o)
+        if pr is None:
+            continue
+        out, err = pr.communicate()
+        if pr.returncode != 0:
+            raise RuntimeError(f"compile of {os.path.basename(src)} failed:\n{err}")
+        if verbose:
+            print(err)
+        logs.append(f"==== {os.path.basename(src)}\n{err}")
+    if logs:
+        with open(os.path.join(bdir, "ptxas.log"), "a") as f:
+            f.write("\n".join(logs))
     tmp = lib + ".tmp"
     cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-Xcompiler", "-fopenmp", "-lgomp"]
     subprocess.check_call(cmd)
     os.replace(tmp, lib)
+    # stamp the library with the build's start time: a source edited while it compiled
+    # makes the next build() recompile
+    os.utime(lib, (t_start, t_start))
     return lib
 
 

@@ -118,6 +118,8 @@ def setup_rank(systems, device: int, mode: str = "alg2", lanes: int = 1, sms: in
                 extra["parts"] = 1 if A.n <= 4096 else min(16, lane_ctas)
             else:
                 extra["parts"] = lane_ctas
+        if device >= 0 and s.K == 0:
+            extra.setdefault("setup", "gpu")      # NEXT-1: ILU(0) setups on the GPU
         h = SPCG(A, mode=mode, K=s.K, device=device, **extra)
         h.lane = lane_of.get(s.index, 0)
         handles.append((s, A, b, h, time.perf_counter() - t0))

@@ -141,21 +141,45 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         h->A.rp.assign(Ain->row_ptr, Ain->row_ptr + Ain->n + 1);
         h->A.col.assign(Ain->col_idx, Ain->col_idx + Ain->nnz);
         h->A.val.assign(Ain->val, Ain->val + Ain->nnz);
-        std::vector<int64_t> pos_t;
-        spcg_status_t st = validate_and_mirror(h->A, pos_t);
-        if (st != SPCG_OK) { delete h; return st; }
-        double t1 = now_ms();
-        st = sparsify_select(h->A, pos_t, drop, h->sp);
-        if (st != SPCG_OK) { delete h; return st; }
-        double t2 = now_ms();
+        if (opt.setup_device < 0 || opt.setup_device > SPCG_SETUP_GPU) {
+            delete h;
+            set_error("bad setup_device");
+            return SPCG_ERR_INVALID_ARG;
+        }
+        const bool on_gpu = opt.setup_device == SPCG_SETUP_GPU && K == 0 && opt.device >= 0;
+        double t1, t2, t3, t4;
+        spcg_status_t st;
+        if (on_gpu) {
+            // NEXT-1: validation, Algorithm 2, ILU(0) and the level sets on the GPU
+            DevAllocator alc;
+            alc.alloc = opt.dev_alloc;
+            alc.free = opt.dev_free;
+            alc.ctx = opt.alloc_ctx;
+            double ph[5] = {0, 0, 0, 0, 0};
+            st = gpu_setup_k0(h->A, drop, opt.device, opt.stream, alc, h->sp, h->F, ph);
+            h->info.zero_pivot_row = h->F.zero_pivot_row;
+            if (st != SPCG_OK) { delete h; return st; }
+            t1 = t0 + ph[0];
+            t2 = t1 + ph[1];
+            t3 = t2 + ph[2];
+            t4 = now_ms();               // ILU(0), factor levels, download of Ahat / L / U
+        } else {
+            std::vector<int64_t> pos_t;
+            st = validate_and_mirror(h->A, pos_t);
+            if (st != SPCG_OK) { delete h; return st; }
+            t1 = now_ms();
+            st = sparsify_select(h->A, pos_t, drop, h->sp);
+            if (st != SPCG_OK) { delete h; return st; }
+            t2 = now_ms();
+            st = iluk_symbolic(h->sp.Ahat, K < 0 ? 0 : K, h->F);
+            if (st != SPCG_OK) { delete h; return st; }
+            t3 = now_ms();
+            st = ilu_numeric(h->sp.Ahat, h->F);
+            h->info.zero_pivot_row = h->F.zero_pivot_row;
+            if (st != SPCG_OK) { delete h; return st; }
+            t4 = now_ms();
+        }
         const Csr& Ah = h->sp.Ahat;
-        st = iluk_symbolic(Ah, K < 0 ? 0 : K, h->F);
-        if (st != SPCG_OK) { delete h; return st; }
-        double t3 = now_ms();
-        st = ilu_numeric(Ah, h->F);
-        h->info.zero_pivot_row = h->F.zero_pivot_row;
-        if (st != SPCG_OK) { delete h; return st; }
-        double t4 = now_ms();
 
         // executor and grid
         int sms = 148;
@@ -197,6 +221,19 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
                     h->lay.C = ChainLayout();
                 } else {
                     chain_ctas = p;
+                }
+            }
+            // AUTO keeps the chain executor where it measured fastest (profiles/r02/exec_cmp):
+            // 2-D chains (components, grid2d; 1024^2 Poisson 2.94 vs 3.17 ms/it chunked); not
+            // 3-D grids, whose z-couplings cross chains through flags (64^3 Poisson 1.06 vs
+            // 0.43 ms/it chunked tiles); and small systems only when every dependency is a
+            // shuffle (else the one-CTA resident executor: 64^2 Poisson 0.089 vs 0.142 ms/it)
+            if (chain_built && strategy == SPCG_SPTRSV_AUTO) {
+                const ChainLayout& CL = h->lay.C;
+                const bool pure = CL.hist_entries + CL.glob_entries + CL.ext_entries == 0;
+                if (CL.partition == "grid3d" || (h->n <= SPCG_RESIDENT_MAX_N && !pure)) {
+                    chain_built = false;
+                    h->lay.C = ChainLayout();
                 }
             }
             if (chain_built) strategy = SPCG_SPTRSV_WCHAIN;
@@ -297,6 +334,7 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         I.sptrsv = strategy;
         I.parts = parts;
         I.device_bytes = bytes;
+        I.setup_device = on_gpu ? SPCG_SETUP_GPU : SPCG_SETUP_HOST;
         {
             static const char* kinds[] = {"contiguous", "strided", "affinity", "components", "tiles"};
             I.partition = -1;
@@ -324,6 +362,7 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             I.algo_bytes_per_iter = 12.0 * (I.nnz_A + I.nnz_L + nU_s) + 8.0 * n + 12.0 * (n + 1) + 8.0 * n + 120.0 * n;
             I.algo_flops_per_iter = 2.0 * (I.nnz_A + I.nnz_L + nU_s) + n + 12.0 * n;
         }
+        I.setup_ms_total = now_ms() - t0;
         *out = h;
         return SPCG_OK;
     } catch (const std::bad_alloc&) {

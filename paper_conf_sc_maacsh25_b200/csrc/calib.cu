@@ -128,6 +128,59 @@ double median(std::vector<double> v) {
     return v[v.size() / 2];
 }
 
+// LL ready-flag stress (DESIGN.md §5.3 "Ready flags"): the executors publish a value
+// as ONE 16-byte store {lo32, epoch, hi32, epoch} (dev_common.cuh ll_store) and accept
+// it when a 16-byte volatile load sees both epochs current — correct only if each
+// 8-byte half {lo32, epoch} / {hi32, epoch} is observed whole.  Producer CTAs rewrite
+// every slot once per epoch with a value both of whose halves encode (epoch, slot);
+// consumer CTAs poll slots at random the whole time.  torn = loads whose two epochs
+// agree but whose value halves do not belong to that epoch (must be 0); mixed = loads
+// whose two epochs differ (benign: the reader keeps spinning).
+__device__ __forceinline__ unsigned ll_lo(unsigned e, unsigned s) { return (e * 0x9E3779B1u) ^ (s * 0x85EBCA77u); }
+__device__ __forceinline__ unsigned ll_hi(unsigned e, unsigned s) { return ~(e * 0xC2B2AE3Du) ^ (s * 0x27D4EB2Fu); }
+
+__global__ void k_llstress(uint4* slots, int nslots, int rounds, unsigned* done, unsigned long long* cnt) {
+    const int nprod = (gridDim.x + 1) / 2;
+    if ((blockIdx.x & 1) == 0) {
+        const int p = blockIdx.x / 2;
+        for (unsigned e = 1; e <= (unsigned)rounds; ++e)
+            for (int s = p * blockDim.x + threadIdx.x; s < nslots; s += nprod * blockDim.x)
+                asm volatile("st.volatile.global.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(slots + s),
+                             "r"(ll_lo(e, (unsigned)s)), "r"(e), "r"(ll_hi(e, (unsigned)s)), "r"(e)
+                             : "memory");
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            atomicAdd(done, 1u);
+        }
+        return;
+    }
+    unsigned long long torn = 0, mixed = 0, ok = 0;
+    unsigned x = 0x12345u + 7919u * (blockIdx.x * blockDim.x + threadIdx.x);
+    for (int it = 0;; ++it) {
+        if ((it & 255) == 0) {
+            unsigned d;
+            asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(d) : "l"(done) : "memory");
+            if (d >= (unsigned)nprod) break;
+        }
+        x = x * 1664525u + 1013904223u;
+        const unsigned s = (x >> 8) % (unsigned)nslots;
+        unsigned a, e1, c, e2;
+        asm volatile("ld.volatile.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(a), "=r"(e1), "=r"(c), "=r"(e2)
+                     : "l"(slots + s)
+                     : "memory");
+        if (e1 != e2) ++mixed;
+        else if (e1 != 0) {
+            if (a != ll_lo(e1, s) || c != ll_hi(e1, s)) ++torn;
+            else ++ok;
+        }
+    }
+    atomicAdd(cnt + 0, torn);
+    atomicAdd(cnt + 1, mixed);
+    atomicAdd(cnt + 2, ok);
+}
+
 }  // namespace
 
 #define CKC(x)                                                            \
@@ -269,5 +322,50 @@ done:
     if (e0) cudaEventDestroy(e0);
     if (e1) cudaEventDestroy(e1);
     if (s) cudaStreamDestroy(s);
+    return st;
+}
+
+extern "C" spcg_status_t spcg_ll_stress(int32_t device, int32_t nslots, int32_t rounds, uint64_t* out) {
+    if (!out || nslots <= 0 || rounds <= 0) {
+        spcg::set_error("spcg_ll_stress: out == NULL or a non-positive size");
+        return SPCG_ERR_INVALID_ARG;
+    }
+    if (cudaSetDevice(device) != cudaSuccess) {
+        spcg::set_error("cudaSetDevice failed");
+        return SPCG_ERR_CUDA;
+    }
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    uint4* slots = nullptr;
+    unsigned* done = nullptr;
+    unsigned long long* cnt = nullptr;
+    spcg_status_t st = SPCG_OK;
+    int G = sms - (sms & 1);            // pairs of producer / consumer CTAs, all co-resident
+    void* args[] = {&slots, &nslots, &rounds, &done, &cnt};
+    if (cudaMalloc(&slots, sizeof(uint4) * (size_t)nslots) != cudaSuccess || cudaMalloc(&done, 4) != cudaSuccess ||
+        cudaMalloc(&cnt, 24) != cudaSuccess) {
+        st = SPCG_ERR_OOM;
+        goto out_;
+    }
+    cudaMemset(slots, 0, sizeof(uint4) * (size_t)nslots);
+    cudaMemset(done, 0, 4);
+    cudaMemset(cnt, 0, 24);
+    if (cudaLaunchCooperativeKernel((void*)k_llstress, dim3(G), dim3(256), args, 0, 0) != cudaSuccess ||
+        cudaDeviceSynchronize() != cudaSuccess) {
+        spcg::set_error(std::string("ll stress kernel: ") + cudaGetErrorString(cudaGetLastError()));
+        st = SPCG_ERR_CUDA;
+        goto out_;
+    }
+    {
+        unsigned long long h[3];
+        cudaMemcpy(h, cnt, 24, cudaMemcpyDeviceToHost);
+        out[0] = h[0];
+        out[1] = h[1];
+        out[2] = h[2];
+    }
+out_:
+    cudaFree(slots);
+    cudaFree(done);
+    cudaFree(cnt);
     return st;
 }

@@ -228,13 +228,16 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
     out.nchains = nch;
     out.chain_step.assign(nch + 1, 0);
     int64_t g = 0;
+    // rows by schedule key (the wavefront level, or the packed component step), rows
+    // ascending inside a key; a key with more than 32 rows spans several steps
+    auto key = [&](int32_t x) -> int64_t { return CP.key.empty() ? (int64_t)F.levL[x] : CP.key[x]; };
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int32_t c = 0; c < CP.nchains; ++c)
+        std::stable_sort(rows.begin() + cstart[c], rows.begin() + cstart[c + 1],
+                         [&](int32_t x, int32_t y) { return key(x) < key(y); });
     for (int32_t c = 0; c < CP.nchains; ++c) {
         if (remap[c] < 0) continue;
         auto b = rows.begin() + cstart[c], e = rows.begin() + cstart[c + 1];
-        // rows by schedule key (the wavefront level, or the packed component step), rows
-        // ascending inside a key; a key with more than 32 rows spans several steps
-        auto key = [&](int32_t x) -> int64_t { return CP.key.empty() ? (int64_t)F.levL[x] : CP.key[x]; };
-        std::stable_sort(b, e, [&](int32_t x, int32_t y) { return key(x) < key(y); });
         out.chain_step[remap[c]] = g;
         for (auto it = b; it != e;) {
             auto jt = it;
@@ -281,9 +284,12 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
         const int rb = upper ? out.rec_U : out.rec_L;
         std::vector<uint8_t>& R = upper ? out.recU : out.recL;
         const size_t trailer = (size_t)384 * W + (upper ? 256 : 0);
+        int64_t n_prev = 0, n_hist = 0, n_glob = 0, n_ext = 0;
+        bool bad = false;
+#pragma omp parallel for schedule(dynamic, 1) reduction(+ : n_prev, n_hist, n_glob, n_ext) reduction(|| : bad)
         for (int32_t c = 0; c < nch; ++c) {
             const int64_t s0 = out.chain_step[c], s1 = out.chain_step[c + 1];
-            for (int64_t s = s0; s < s1; ++s) {
+            for (int64_t s = s0; s < s1 && !bad; ++s) {
                 uint32_t flags = 0;
                 const size_t base = (size_t)s * rb;
                 for (int l = 0; l < 32; ++l) {
@@ -302,20 +308,22 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
                             const int64_t sj = pj / 32;
                             const int64_t ps_j = upper ? (s1 - 1 - sj) : (sj - s0);
                             const int64_t d = ps_i - ps_j;
-                            if (d < 1) { if (why) *why = "internal: dependency not earlier in its chain"; return false; }
+                            if (d < 1) { bad = true; break; }
                             if (d == 1) {
                                 tag = ((uint32_t)CT_PREV << 29) | (uint32_t)(pj & 31);
-                                out.prev_entries++;
+                                n_prev++;
                             } else if (d < SPCG_CHAIN_HIST) {
                                 tag = ((uint32_t)CT_HIST << 29) | (uint32_t)(pj & 31) | ((uint32_t)d << 5);
                                 flags |= CS_SLOW;
-                                out.chain_flags[c] |= upper ? CC_UHIST : CC_LHIST;
-                                out.hist_entries++;
+                                __atomic_fetch_or(&out.chain_flags[c], (uint32_t)(upper ? CC_UHIST : CC_LHIST),
+                                                  __ATOMIC_RELAXED);
+                                n_hist++;
                             } else {
                                 tag = ((uint32_t)CT_GLOB << 29) | (uint32_t)pj;
                                 flags |= CS_SLOW;
-                                out.chain_flags[c] |= upper ? CC_UGLOB : CC_LGLOB;
-                                out.glob_entries++;
+                                __atomic_fetch_or(&out.chain_flags[c], (uint32_t)(upper ? CC_UGLOB : CC_LGLOB),
+                                                  __ATOMIC_RELAXED);
+                                n_glob++;
                             }
                         } else {
                             if (next < 2) {
@@ -325,27 +333,33 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
                                 tag = ((uint32_t)CT_EXTS << 29) | (uint32_t)pj;
                             }
                             flags |= CS_SLOW | CS_EXT;
-                            out.chain_flags[c] |= upper ? CC_UEXT : CC_LEXT;
-                            out.chain_flags[cj] |= upper ? CC_UPUB : CC_LPUB;
-                            out.ext_entries++;
-                            // the producer publishes its value with a ready flag
+                            __atomic_fetch_or(&out.chain_flags[c], (uint32_t)(upper ? CC_UEXT : CC_LEXT),
+                                              __ATOMIC_RELAXED);
+                            __atomic_fetch_or(&out.chain_flags[cj], (uint32_t)(upper ? CC_UPUB : CC_LPUB),
+                                              __ATOMIC_RELAXED);
+                            n_ext++;
+                            // the producer publishes its value with a ready flag (its record's
+                            // trailer: 4-byte aligned, possibly another chain's -> atomic OR)
                             const int64_t sj = pj / 32;
                             const size_t pb = (size_t)sj * rb + trailer;
-                            uint32_t m;
-                            std::memcpy(&m, R.data() + pb, 4);
-                            m |= 1u << (pj & 31);
-                            std::memcpy(R.data() + pb, &m, 4);
+                            __atomic_fetch_or((uint32_t*)(R.data() + pb), 1u << (pj & 31), __ATOMIC_RELAXED);
                         }
                         put<uint32_t>(R, base + 4 * ((size_t)W * l + k), tag);
                         put<double>(R, base + (size_t)128 * W + 8 * ((size_t)W * l + k), M.val[q]);
                     }
                     if (upper) put<double>(R, base + (size_t)384 * W + 8 * l, 1.0 / M.val[M.rp[i]]);
                 }
-                uint32_t f0;
-                std::memcpy(&f0, R.data() + base + trailer + 4, 4);
-                put<uint32_t>(R, base + trailer + 4, f0 | flags);
+                __atomic_fetch_or((uint32_t*)(R.data() + base + trailer + 4), flags, __ATOMIC_RELAXED);
             }
         }
+        if (bad) {
+            if (why) *why = "internal: dependency not earlier in its chain";
+            return false;
+        }
+        out.prev_entries += n_prev;
+        out.hist_entries += n_hist;
+        out.glob_entries += n_glob;
+        out.ext_entries += n_ext;
     }
 
     // SpMV: SELL-32 of the ORIGINAL A over positions, one slice per step;
@@ -362,6 +376,7 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
     for (int64_t s = 0; s < g; ++s) S.eoff[s + 1] = S.eoff[s] + WA;
     S.col.assign(S.eoff[g] * 32, 0);
     S.val.assign(S.eoff[g] * 32, 0.0);
+#pragma omp parallel for schedule(static)
     for (int64_t s = 0; s < g; ++s)
         for (int l = 0; l < 32; ++l) {
             const int32_t i = out.perm[32 * s + l];
@@ -405,8 +420,9 @@ bool chain_smem_config(const ChainLayout& CL, int per_cta, ChainSmemCfg& out) {
             out.hist_off = (uint32_t)hist_off;
             out.cta_bytes = warp * per_cta;
             // SpMV staging (the same shared memory, used between the triangular solves):
-            // 8 warps x sp_nst stages of SPCG_SPMV_G slices of WA entry columns
-            const size_t sp_stage = (size_t)SPCG_SPMV_G * CL.WA * 384;
+            // 8 warps x sp_nst stages of SPCG_SPMV_G slices of WA entry columns, plus two
+            // operand windows of SPCG_SPMV_G + 2 halo slices (p_old and z, wchain.cu)
+            const size_t sp_stage = (size_t)SPCG_SPMV_G * CL.WA * 384 + 2 * (size_t)(SPCG_SPMV_G + 2) * 256;
             out.sp_nst = 0;
             out.sp_stage_bytes = (uint32_t)sp_stage;
             for (int sn = 3; sn >= 2; --sn)

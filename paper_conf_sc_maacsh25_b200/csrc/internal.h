@@ -7,6 +7,8 @@
 
 #include "../../include/spcg.h"
 
+struct DevAllocator;               // spcg_options_t allocator hooks (defined below)
+
 namespace spcg {
 
 struct Csr {                       // host CSR, int64 row pointers
@@ -53,6 +55,14 @@ struct Factors {
 };
 spcg_status_t iluk_symbolic(const Csr& Ahat, int K, Factors& F);
 spcg_status_t ilu_numeric(const Csr& Ahat, Factors& F);
+
+// ---- gsetup.cu (NEXT-1) ------------------------------------------------------
+// Validation, Algorithm 2, ILU(0) and the factor level sets on the GPU; fills sp and F
+// exactly as validate_and_mirror + sparsify_select + iluk_symbolic(K = 0) + ilu_numeric
+// do (bit-exact; the Frobenius indicator values up to summation order).  phase_ms[5]:
+// upload + validation, Algorithm 2, L/U split, ILU(0) + levels, download.
+spcg_status_t gpu_setup_k0(const Csr& A, const spcg_drop_params_t& p, int device, void* stream,
+                           const ::DevAllocator& alc, SparsifyResult& sp, Factors& F, double* phase_ms);
 
 // ---- layout.cpp ------------------------------------------------------------
 // Sliced-ELL (slice height 32, column-major inside a slice) triangular-solve
@@ -214,7 +224,7 @@ void build_tri_layouts(const Factors& F, int strategy, int parts, int ring_max, 
 struct spcg_device_s;
 typedef struct spcg_device_s spcg_device_t;
 
-struct DevAllocator {               // spcg_options_t allocator hooks (NULL: cudaMalloc / cudaFree)
+struct DevAllocator {         // spcg_options_t allocator hooks (NULL: cudaMalloc / cudaFree)
     spcg_dev_alloc_fn alloc = nullptr;
     spcg_dev_free_fn free = nullptr;
     void* ctx = nullptr;

@@ -1670,6 +1670,7 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         AL(vb, P.CH.xp, double*);
         AL(vb, P.CH.bp, double*);
         AL(vb, P.CH.t1, double*);
+        AL(vb, P.CH.p2, double*);
     }
     AL(d->mb_bytes, P.mbL, uint4*);
     AL(d->mb_bytes, P.mbU, uint4*);

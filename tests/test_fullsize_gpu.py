@@ -69,9 +69,29 @@ def test_full_size_alg2(name):
     L, U, info = oracle.setup(A, mode="alg2", K=K)
     h = lib.SPCG(A, mode="alg2", K=K)
     check_setup_bit_exact(h, A, info["Ahat"], L, U, info["fill_level"], info)
+    if K == 0:
+        _gpu_setup_same_products(A, h, info)
     _operators_all_rows(h, A, L, U)
     _full_solve_parity(h, A, b, L, U)
     h.close()
+
+
+def _gpu_setup_same_products(A, h, info):
+    """NEXT-1 at full size: the GPU setup (gsetup.cu) yields the host setup's products bit
+    for bit (the host handle h is itself checked against the oracle above); the Frobenius
+    indicators agree with the oracle's up to summation order (reading A6g: 2 (N-1) 2^-53
+    per sum, N = nnz(A) terms)."""
+    hg = lib.SPCG(A, mode="alg2", K=0, setup="gpu")
+    assert hg.info["setup_device"] == 1
+    for e in ("ahat_rowptr", "ahat_col", "ahat_val", "l_rowptr", "l_col", "l_val", "u_rowptr", "u_col", "u_val",
+              "level_l", "level_u", "levelrows_l", "levelrows_u"):
+        assert np.array_equal(hg.export(e).view(np.uint8), h.export(e).view(np.uint8)), e
+    for k in ("chosen_pct", "m_t", "w_A", "w_Ahat", "n_tried", "tried_w", "levels_L", "levels_U"):
+        assert hg.info[k] == h.info[k], k
+    tol = 8.0 * A.nnz * 2.0 ** -53
+    for r, x in enumerate(info["trace"]):
+        assert abs(hg.info["indicator"][r] - x["ind"]) <= tol * abs(x["ind"]), (r, hg.info["indicator"][r], x)
+    hg.close()
 
 
 @pytest.mark.parametrize("name", ["C1", "C2"])

@@ -176,6 +176,17 @@ def test_calibrate_handoffs_are_ordered():
     assert c["flag_same_die_ns"] < c["grid_sync_ns"]
 
 
+def test_ll_flags_never_tear():
+    """Robustness of the 16-byte LL ready flags {lo32, epoch, hi32, epoch} (DESIGN.md
+    §5.3): under concurrent rewrites from half the SMs and random polling from the
+    other half, no load ever sees both epochs current with a value from another epoch.
+    Small slot counts put producer and consumers on the same lines constantly."""
+    for nslots, rounds in ((64, 20000), (4096, 2000), (1 << 20, 20)):
+        r = lib.ll_stress(0, nslots, rounds)
+        assert r["torn"] == 0, (nslots, rounds, r)
+        assert r["ok"] > 0, r
+
+
 def test_async_concurrent_solves_match_sync():
     """spcg_solve_async / spcg_solve_wait: independent systems in flight on separate
     streams (C5 lanes) give bitwise the results of spcg_solve."""

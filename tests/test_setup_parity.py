@@ -27,7 +27,7 @@ def test_library_exports_every_declared_symbol():
     for name in declared:
         assert hasattr(L, name), name
     assert declared == set(lib.EXPORTED)
-    assert L.spcg_abi_version() == 2
+    assert L.spcg_abi_version() == 3
 
 
 CASES = [

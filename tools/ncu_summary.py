@@ -24,6 +24,8 @@ def main():
     ap.add_argument("--workload", default="C2"); ap.add_argument("--impl", default="spcg")
     ap.add_argument("--json", default="profiles/ncu_summary.json")
     ap.add_argument("--note", default="")
+    ap.add_argument("--iterations", type=int, default=0,
+                    help="forced-k iterations of the captured launch (per-iteration DRAM bytes = launch / (k + 1))")
     a = ap.parse_args()
     h, units, data = raw(a.rep)
     lines = [f"# ncu summary — {a.workload} ({a.impl})", "", a.note, "", f"report: `{os.path.basename(a.rep)}` (ncu --set full --clock-control none)", ""]
@@ -70,8 +72,13 @@ def main():
     rd = float(d["dram__bytes_read.sum"][0]) * UNIT.get(d["dram__bytes_read.sum"][1], 1)
     wr = float(d["dram__bytes_write.sum"][0]) * UNIT.get(d["dram__bytes_write.sum"][1], 1)
     js = json.load(open(a.json)) if os.path.exists(a.json) else {}
-    js.setdefault(a.workload, {})[a.impl] = {"dram_bytes_per_launch": rd + wr, "report": os.path.basename(a.rep),
-                                           "summary": os.path.basename(a.out)}
+    e = {"dram_bytes_per_launch": rd + wr, "report": os.path.basename(a.rep), "summary": os.path.basename(a.out)}
+    if a.iterations > 0:
+        e["iterations_in_launch"] = a.iterations
+        e["dram_bytes_per_iter"] = (rd + wr) / (a.iterations + 1)
+    if "lts__t_sector_hit_rate.pct" in d:
+        e["l2_hit_pct"] = float(d["lts__t_sector_hit_rate.pct"][0])
+    js.setdefault(a.workload, {})[a.impl] = e
     json.dump(js, open(a.json, "w"), indent=1)
     print(open(a.out).read())
 
