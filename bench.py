@@ -216,6 +216,7 @@ def main():
     ap.add_argument("--parts", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-host-setup", action="store_true", help="skip timing the host setup beside the GPU one")
+    ap.add_argument("--no-f32", action="store_true", help="skip the fp32-factor (NEXT-2) leg of C4")
     ap.add_argument("--batch-count", type=int, default=64)
     ap.add_argument("--lanes", type=int, default=4,
                     help="C5: concurrent streams per GPU (each with SMs/lanes persistent CTAs)")
@@ -335,6 +336,25 @@ def main():
                       "hbm_gbs_per_iter": hs.info["algo_bytes_per_iter"] * tk / (float(np.mean(tms)) * 1e-3) / 1e9})
         hs.close()
 
+    # NEXT-2: fp32 factors with fp64 vectors (the paper's preconditioner precision,
+    # P:L827-828) on the same workload: M = fl32(L) fl32(U), 4-byte record values
+    f32 = None
+    if name == "C4" and not args.no_f32:
+        hf = spcg.SPCG(A, mode="alg2", K=K, sptrsv=args.sptrsv, parts=args.parts, device=dev, stream=stream,
+                       setup=setup_kind, factors="f32")
+        hf.solve(bd, xd, EPS, KMAX)
+        fms, fk = [], 0
+        for _ in range(max(1, min(args.steps, 3))):
+            flush.zero_()
+            _, inf = hf.solve(bd, xd, EPS, KMAX)
+            fms.append(inf["iter_phase_ms"])
+            fk = inf["iterations"]
+        fb = hf.info["algo_bytes_per_iter"]
+        f32 = {"ms": float(np.mean(fms)), "iterations": fk, "ms_per_iter": float(np.mean(fms)) / max(fk, 1),
+               "algo_bytes_per_iter": fb, "record_value_bytes": hf.info["record_value_bytes"],
+               "hbm_gbs_per_iter": fb * fk / (float(np.mean(fms)) * 1e-3) / 1e9, "status": inf["status"]}
+        hf.close()
+
     def mx(v):
         if ws == 1:
             return v
@@ -385,6 +405,8 @@ def main():
         "pcg": {"value": p_ms, "iterations": p["k"], "ms_per_iter": p_ms / max(p["k"], 1), "hbm_gbs_per_iter": p_gbs,
                 "algo_bytes_per_iter": p_bi, "levels": {"L": pi["levels_L"], "U": pi["levels_U"]}},
         "sweep": sweep or None,
+        "fp32_factors": None if f32 is None else dict(f32, frac=f32["hbm_gbs_per_iter"] / peak,
+                                                       note="NEXT-2: M = fl32(L) fl32(U) applied in fp64"),
         "spcg_vs_pcg": {"iter_phase_speedup": p_ms / s_ms,
                         "per_iter_speedup": (p_ms / max(p["k"], 1)) / (s_ms / max(s["k"], 1))},
         "paper_context": PAPER_CONTEXT,

@@ -48,7 +48,8 @@ enum {
     SPCG_ERR_INVALID_ARG = -1,
     SPCG_ERR_BAD_MATRIX = -2,   /* non-square, unsorted/duplicate cols, missing or <= 0 diagonal,
                                    non-finite value, not exactly (bitwise) symmetric, nnz >= 2^31 */
-    SPCG_ERR_ZERO_PIVOT = -3,   /* u_ii == 0 or non-finite during ILU (row in setup info) */
+    SPCG_ERR_ZERO_PIVOT = -3,   /* u_ii == 0 or non-finite during ILU, or after rounding to fp32
+                                   (row in setup info) */
     SPCG_ERR_BREAKDOWN = -4,    /* (p,w) <= 0 or a non-finite PCG scalar */
     SPCG_ERR_OOM = -5,
     SPCG_ERR_CUDA = -6,
@@ -112,6 +113,7 @@ enum {
 };
 
 enum { SPCG_SETUP_HOST = 0, SPCG_SETUP_GPU = 1 };
+enum { SPCG_FACTORS_F64 = 0, SPCG_FACTORS_F32 = 1 };
 
 /* Device allocator hooks: when dev_alloc is set, every device buffer the handle owns
  * comes from dev_alloc(bytes, stream, ctx) and goes back through
@@ -142,7 +144,12 @@ typedef struct {
                                    K = -1 run on the host).  Products are bit-exact with the host setup
                                    except the Frobenius indicator values, which agree up to summation
                                    order (reading A6g) */
-    int32_t reserved[6];
+    int32_t factor_precision;   /* SPCG_FACTORS_F64 (default) or SPCG_FACTORS_F32 (NEXT-2, the paper's
+                                   fp32 preconditioner): the ILU factor values are rounded to
+                                   fp32 after the factorisation, M = fl32(L) fl32(U) applied in fp64
+                                   (1/u_ii from the rounded u_ii); the warp-chain records then carry
+                                   4-byte values.  Vectors and scalars stay fp64, so eps = 1e-8 holds */
+    int32_t reserved[5];
 } spcg_options_t;
 
 typedef struct {
@@ -174,6 +181,8 @@ typedef struct {
     int64_t chain_entries[4];   /* WCHAIN: dependencies read by shuffle / shared ring / global / flag */
     int32_t setup_device;       /* where validation .. ILU ran: SPCG_SETUP_HOST / SPCG_SETUP_GPU */
     double setup_ms_total;      /* spcg_setup wall time, entry to return */
+    int32_t factor_precision;   /* SPCG_FACTORS_*: precision of the stored factor values */
+    int32_t record_value_bytes; /* WCHAIN: bytes per stored factor value in the records (8 or 4) */
 } spcg_setup_info_t;
 
 typedef struct {

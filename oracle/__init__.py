@@ -251,6 +251,15 @@ def setup(A: CSR, mode: str = "alg2", K: int = 0, fixed_pct: float = 0.0, **alg2
     return L, U, info
 
 
+def round_factors_f32(L: CSR, U: CSR):
+    """NEXT-2: the paper's fp32 preconditioner applied in fp64 — every stored
+    factor value rounded to the nearest fp32 (IEEE round to nearest even, as a C
+    (float) cast), the operator M = fl32(L) fl32(U).  Returns new CSRs."""
+    def r(M):
+        return CSR(M.n, M.row_ptr, M.col, M.val.astype(np.float32).astype(np.float64), M.name)
+    return r(L), r(U)
+
+
 # ---------------------------------------------------------------- multicore baseline
 _OMP_SRC = os.path.join(_HERE, "spcg_oracle_omp.c")
 _OMP_LIB = os.path.join(_HERE, "liboracle_omp.so")

@@ -77,7 +77,8 @@ class Options(ctypes.Structure):
                 ("parts", ctypes.c_int32), ("host_threads", ctypes.c_int32), ("exec", ctypes.c_int32),
                 ("dev_alloc", _ALLOC_FN), ("dev_free", _FREE_FN), ("alloc_ctx", ctypes.c_void_p),
                 ("wide_min", ctypes.c_double), ("chunk_partition", ctypes.c_int32),
-                ("setup_device", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
+                ("setup_device", ctypes.c_int32), ("factor_precision", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 5)]
 
 
 class SetupInfo(ctypes.Structure):
@@ -94,7 +95,8 @@ class SetupInfo(ctypes.Structure):
                 ("algo_bytes_per_iter", ctypes.c_double), ("algo_flops_per_iter", ctypes.c_double),
                 ("partition", ctypes.c_int32), ("chains", ctypes.c_int32), ("positions", ctypes.c_int64),
                 ("chain_entries", ctypes.c_int64 * 4), ("setup_device", ctypes.c_int32),
-                ("setup_ms_total", ctypes.c_double)]
+                ("setup_ms_total", ctypes.c_double), ("factor_precision", ctypes.c_int32),
+                ("record_value_bytes", ctypes.c_int32)]
 
 
 class SolveInfo(ctypes.Structure):
@@ -245,11 +247,13 @@ class SPCG:
     allocator: "torch" (default: device buffers from PyTorch's caching allocator through
     the spcg_options_t hooks) or "cuda" (the library's own cudaMalloc).
     setup: "host" (default) or "gpu" (NEXT-1: validation, Algorithm 2, ILU(0) and the
-    level sets on the device; K = 0 only, other K run on the host)."""
+    level sets on the device; K = 0 only, other K run on the host).
+    factors: "f64" (default) or "f32" (NEXT-2: factor values rounded to fp32, the paper's
+    preconditioner precision; vectors stay fp64)."""
 
     def __init__(self, A, mode="alg2", K=0, fixed_pct=0.0, sptrsv="auto", parts=0, device=0, stream=None,
                  host_threads=0, allocator="torch", exec="auto", wide_min=0.0, chunk_partition=-1, setup="host",
-                 **drop_kw):
+                 factors="f64", **drop_kw):
         lib = load()
         rp = np.ascontiguousarray(A.row_ptr, np.int64)
         col = np.ascontiguousarray(A.col, np.int32)
@@ -267,6 +271,7 @@ class SPCG:
         opt.wide_min = wide_min
         opt.chunk_partition = chunk_partition
         opt.setup_device = {"host": 0, "gpu": 1}[setup]
+        opt.factor_precision = {"f64": 0, "f32": 1}[factors]
         self.device = device
         self._alloc = None
         if device >= 0:

@@ -180,6 +180,33 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             t4 = now_ms();
         }
         const Csr& Ah = h->sp.Ahat;
+        // NEXT-2: fp32 factors: round every stored L / U value to fp32 (IEEE
+        // round to nearest even); the operator is M = fl32(L) fl32(U), applied in fp64
+        if (opt.factor_precision < 0 || opt.factor_precision > SPCG_FACTORS_F32) {
+            delete h;
+            set_error("bad factor_precision");
+            return SPCG_ERR_INVALID_ARG;
+        }
+        if (opt.factor_precision == SPCG_FACTORS_F32 && !h->identity) {
+            for (double& v : h->F.L.val) v = (double)(float)v;
+            for (double& v : h->F.U.val) v = (double)(float)v;
+            for (int64_t i = 0; i < h->n; ++i) {
+                const double d = h->F.U.val[h->F.U.rp[i]];
+                if (d == 0.0 || !std::isfinite(d)) {
+                    h->info.zero_pivot_row = i;
+                    delete h;
+                    set_error("pivot u_ii rounds to 0 or overflows in fp32 at row " + std::to_string(i));
+                    return SPCG_ERR_ZERO_PIVOT;
+                }
+            }
+            for (double v : h->F.L.val)
+                if (!std::isfinite(v)) {
+                    delete h;
+                    set_error("a factor value overflows fp32");
+                    return SPCG_ERR_INVALID_ARG;
+                }
+        }
+        const bool f32 = opt.factor_precision == SPCG_FACTORS_F32 && !h->identity;
 
         // executor and grid
         int sms = 148;
@@ -204,7 +231,7 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         if ((strategy == SPCG_SPTRSV_AUTO || strategy == SPCG_SPTRSV_WCHAIN) && !h->identity) {
             // components are packed onto as many chains as there are SMs (or the CTAs asked for)
             const int target = opt.parts > 0 ? opt.parts : sms;
-            chain_built = build_chain_layout(h->A, h->F, std::max(1, target), h->lay.C, &chain_why);
+            chain_built = build_chain_layout(h->A, h->F, std::max(1, target), f32, h->lay.C, &chain_why);
             if (chain_built) {
                 // CTAs: one per chain up to the SM count (more chains share CTAs, one solver
                 // warp each); large systems take every SM so the SpMV and vector phases use
@@ -335,6 +362,8 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
         I.parts = parts;
         I.device_bytes = bytes;
         I.setup_device = on_gpu ? SPCG_SETUP_GPU : SPCG_SETUP_HOST;
+        I.factor_precision = f32 ? SPCG_FACTORS_F32 : SPCG_FACTORS_F64;
+        I.record_value_bytes = strategy == SPCG_SPTRSV_WCHAIN ? h->lay.C.vb : 8;
         {
             static const char* kinds[] = {"contiguous", "strided", "affinity", "components", "tiles"};
             I.partition = -1;
@@ -359,7 +388,10 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             I.algo_bytes_per_iter = 12.0 * I.nnz_A + 4.0 * (n + 1) + 96.0 * n;
             I.algo_flops_per_iter = 2.0 * I.nnz_A + 10.0 * n;
         } else {
-            I.algo_bytes_per_iter = 12.0 * (I.nnz_A + I.nnz_L + nU_s) + 8.0 * n + 12.0 * (n + 1) + 8.0 * n + 120.0 * n;
+            // NEXT-2: 4-byte factor values where the records carry them (8 B per entry)
+            const double fb = I.record_value_bytes == 4 ? 8.0 : 12.0;
+            I.algo_bytes_per_iter = 12.0 * I.nnz_A + fb * (I.nnz_L + nU_s) + 8.0 * n + 12.0 * (n + 1) + 8.0 * n +
+                                    120.0 * n;
             I.algo_flops_per_iter = 2.0 * (I.nnz_A + I.nnz_L + nU_s) + n + 12.0 * n;
         }
         I.setup_ms_total = now_ms() - t0;

@@ -192,7 +192,8 @@ void put(std::vector<uint8_t>& b, size_t off, T v) { std::memcpy(b.data() + off,
 
 }  // namespace
 
-bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, ChainLayout& out, std::string* why) {
+bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, bool f32, ChainLayout& out,
+                        std::string* why) {
     const int64_t n = F.L.n;
     out = ChainLayout();
     // dependency columns per record
@@ -271,8 +272,12 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
     auto pow2 = [](int64_t w) { int64_t p = 1; while (p < w) p <<= 1; return (int32_t)p; };
     out.W_L = pow2(std::max<int64_t>(wl, 1));
     out.W_U = pow2(std::max<int64_t>(wu, 1));
-    out.rec_L = 384 * out.W_L + 16;
-    out.rec_U = 384 * out.W_U + 256 + 16;
+    // NEXT-2: fp32 factor values (exactly representable after the setup's rounding) are
+    // stored in 4 bytes when the records are narrow (the kernel's fp32 record variants)
+    out.vb = (f32 && out.W_L <= 4 && out.W_U <= 4) ? 4 : 8;
+    const int vrow = 128 + 32 * out.vb;   // bytes per entry column of a record: tags + values
+    out.rec_L = vrow * out.W_L + 16;
+    out.rec_U = vrow * out.W_U + 256 + 16;
     out.recL.assign((size_t)g * out.rec_L, 0);
     out.recU.assign((size_t)g * out.rec_U, 0);
     out.chain_flags.assign(nch, 0u);
@@ -283,7 +288,7 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
         const int W = upper ? out.W_U : out.W_L;
         const int rb = upper ? out.rec_U : out.rec_L;
         std::vector<uint8_t>& R = upper ? out.recU : out.recL;
-        const size_t trailer = (size_t)384 * W + (upper ? 256 : 0);
+        const size_t trailer = (size_t)vrow * W + (upper ? 256 : 0);
         int64_t n_prev = 0, n_hist = 0, n_glob = 0, n_ext = 0;
         bool bad = false;
 #pragma omp parallel for schedule(dynamic, 1) reduction(+ : n_prev, n_hist, n_glob, n_ext) reduction(|| : bad)
@@ -345,9 +350,12 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, Chain
                             __atomic_fetch_or((uint32_t*)(R.data() + pb), 1u << (pj & 31), __ATOMIC_RELAXED);
                         }
                         put<uint32_t>(R, base + 4 * ((size_t)W * l + k), tag);
-                        put<double>(R, base + (size_t)128 * W + 8 * ((size_t)W * l + k), M.val[q]);
+                        if (out.vb == 4)
+                            put<float>(R, base + (size_t)128 * W + 4 * ((size_t)W * l + k), (float)M.val[q]);
+                        else
+                            put<double>(R, base + (size_t)128 * W + 8 * ((size_t)W * l + k), M.val[q]);
                     }
-                    if (upper) put<double>(R, base + (size_t)384 * W + 8 * l, 1.0 / M.val[M.rp[i]]);
+                    if (upper) put<double>(R, base + (size_t)vrow * W + 8 * l, 1.0 / M.val[M.rp[i]]);
                 }
                 __atomic_fetch_or((uint32_t*)(R.data() + base + trailer + 4), flags, __ATOMIC_RELAXED);
             }
@@ -420,9 +428,8 @@ bool chain_smem_config(const ChainLayout& CL, int per_cta, ChainSmemCfg& out) {
             out.hist_off = (uint32_t)hist_off;
             out.cta_bytes = warp * per_cta;
             // SpMV staging (the same shared memory, used between the triangular solves):
-            // 8 warps x sp_nst stages of SPCG_SPMV_G slices of WA entry columns, plus two
-            // operand windows of SPCG_SPMV_G + 2 halo slices (p_old and z, wchain.cu)
-            const size_t sp_stage = (size_t)SPCG_SPMV_G * CL.WA * 384 + 2 * (size_t)(SPCG_SPMV_G + 2) * 256;
+            // 8 warps x sp_nst stages of SPCG_SPMV_G slices of WA entry columns
+            const size_t sp_stage = (size_t)SPCG_SPMV_G * CL.WA * 384;
             out.sp_nst = 0;
             out.sp_stage_bytes = (uint32_t)sp_stage;
             for (int sn = 3; sn >= 2; --sn)

@@ -71,6 +71,7 @@ struct DevChain {
     int32_t nchains, per_cta;      // chains, solver warps per CTA (chain c -> CTA c % grid, warp c / grid)
     int32_t nst;                   // stages per solver warp (SPCG_CHAIN_C steps each)
     int32_t W_L, W_U, rec_L, rec_U;
+    int32_t vb;                    // bytes per factor value in the records (8, or 4: fp32 factors)
     int32_t any_ext, any_hist;
     uint32_t stage_bytes, warp_bytes, ext_off, hist_off;
     int32_t WA, sp_nst;            // SpMV: uniform slice width, TMA stages per warp (0: register path)

@@ -148,8 +148,9 @@ struct ChunkStream {
 // Algorithm 1 live in execution ("position") order pos = 32 * global_step + lane for
 // the whole solve; b and x are permuted on entry and exit.  A record per step holds,
 // lane-major, W (a power of two) dependency tags + values (and 1/u_ii for U):
-//   tag u32 [32][W] at 0, value f64 [32][W] at 128 W, (U) 1/u_ii f64 [32] at 384 W,
-//   trailer {u32 publish mask (lanes whose value another chain reads), u32 flags}.
+//   tag u32 [32][W] at 0, value f64 [32][W] (f32 with vb = 4) at 128 W, (U) 1/u_ii f64
+//   [32] at (128 + 32 vb) W, trailer {u32 publish mask (lanes whose value another chain
+//   reads), u32 flags}.
 //   tag = kind << 29 | payload:
 //     PREV (0): payload = the lane whose previous-step value is the dependency (a warp
 //               shuffle, no memory access); padding entries are PREV lane 0, value 0
@@ -171,6 +172,7 @@ struct ChainLayout {
     int32_t nchains = 0;
     int32_t W_L = 0, W_U = 0;
     int32_t rec_L = 0, rec_U = 0;         // bytes per record
+    int32_t vb = 8;                       // bytes per factor value in the records (8, or 4 with fp32 factors)
     int64_t nsteps = 0;                   // global steps; positions = 32 * nsteps
     std::vector<int64_t> chain_step;      // [nchains+1] first global step of each chain
     std::vector<uint32_t> chain_flags;    // [nchains] CC_*
@@ -184,12 +186,18 @@ struct ChainLayout {
 };
 // Builds the chain layout when the factors suit it (dependency columns <= WMAX, a
 // partition into chains found); returns false (why set) otherwise.
-bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, ChainLayout& out, std::string* why);
+// f32: the factor values are fp32-representable (NEXT-2) -> 4-byte record values when
+// the records are narrow (W <= 4; wider records keep 8-byte values).
+bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, bool f32, ChainLayout& out,
+                        std::string* why);
 
 // Shared memory of the warp-chain kernel per solver warp: mbarriers (128 B), NST stages
 // of SPCG_CHAIN_C steps (records + the pass's operand slices), the prefetched-flag queue,
 // the history ring.  The most stages (2..16) whose per-CTA total fits; false if none.
-constexpr int SPCG_CHAIN_C = 8;                  // steps per stage (compile-time in the kernel)
+#ifndef SPCG_CHAIN_STEPS
+#define SPCG_CHAIN_STEPS 8
+#endif
+constexpr int SPCG_CHAIN_C = SPCG_CHAIN_STEPS;   // steps per stage (compile-time in the kernel)
 struct ChainSmemCfg {
     int32_t nst = 0;
     uint32_t stage_bytes = 0, warp_bytes = 0, ext_off = 0, hist_off = 0;

@@ -1623,6 +1623,7 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         D.W_U = CL.W_U;
         D.rec_L = CL.rec_L;
         D.rec_U = CL.rec_U;
+        D.vb = CL.vb;
         D.nsteps = CL.nsteps;
         D.npos = nv;
         spcg::ChainSmemCfg cfg;

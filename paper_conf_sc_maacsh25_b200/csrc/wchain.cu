@@ -129,6 +129,27 @@ __device__ __forceinline__ void lds_vals(const uint8_t* __restrict__ p, double (
     }
 }
 
+// fp32 record values (NEXT-2): W floats of this lane, widened exactly to fp64
+template <int W>
+__device__ __forceinline__ void lds_vals_f32(const uint8_t* __restrict__ p, double (&v)[W]) {
+    if constexpr (W == 1) {
+        v[0] = (double)*(const float*)p;
+    } else if constexpr (W == 2) {
+        const float2 a = *(const float2*)p;
+        v[0] = (double)a.x;
+        v[1] = (double)a.y;
+    } else {
+#pragma unroll
+        for (int j = 0; j < W; j += 4) {
+            const float4 a = *(const float4*)(p + 4 * j);
+            v[j] = (double)a.x;
+            v[j + 1] = (double)a.y;
+            v[j + 2] = (double)a.z;
+            v[j + 3] = (double)a.w;
+        }
+    }
+}
+
 // What a GENERAL pass needs besides the shuffle path (HIST / GLOB / EXT entries,
 // published values, the history ring).
 struct GenCtx {
@@ -152,13 +173,14 @@ struct GenCtx {
 // L (KIND K_ITER): ops r, w, x, p: r_i = r - alpha w, x_i = x + alpha p (Alg. 1 lines
 // 11-12 fused), y_i = r_i - sum_k l_ik y_k, ||r||^2;  K_PRO: ops rsrc; K_APPLY: ops in.
 // U: ops y [, rdot]: z_i = (y_i - sum_k u_ik z_k) / u_ii, (rdot, z); K_PRO also p0 = z0.
-template <int W, bool UPPER, int KIND, bool GEN, bool SPLIT, int CNT>
+template <int W, bool UPPER, int KIND, bool GEN, bool SPLIT, int CNT, int VB>
 __device__ __forceinline__ void run_chunk(uint8_t* __restrict__ st, int cnt_rt, int64_t glo, int u0, int nv,
                                           bool rsrc_is_r, int use_x0, double* __restrict__ out,
                                           double* __restrict__ Er, double* __restrict__ Exp, double* __restrict__ Ep,
                                           double alpha, double& yprev, double& dot, const GenCtx& G) {
-    constexpr int RECB = 384 * W + (UPPER ? 256 : 0) + 16;
-    constexpr size_t TRAILER = (size_t)384 * W + (UPPER ? 256 : 0);
+    constexpr int VROW = 128 + 32 * VB;                    // record bytes per entry column
+    constexpr int RECB = VROW * W + (UPPER ? 256 : 0) + 16;
+    constexpr size_t TRAILER = (size_t)VROW * W + (UPPER ? 256 : 0);
     const int lane = threadIdx.x & 31;
     const int cnt = CNT > 0 ? CNT : cnt_rt;
     double* __restrict__ sv = (double*)(st + (size_t)CC * RECB) + lane;
@@ -171,7 +193,8 @@ __device__ __forceinline__ void run_chunk(uint8_t* __restrict__ st, int cnt_rt, 
         uint32_t tg[W];
         double v[W];
         lds_tags<W>(R + 4 * W * lane, tg);
-        lds_vals<W>(R + 128 * W + 8 * W * lane, v);
+        if constexpr (VB == 4) lds_vals_f32<W>(R + 128 * W + 4 * W * lane, v);
+        else lds_vals<W>(R + 128 * W + 8 * W * lane, v);
         double acc, ri = 0.0, xn = 0.0, rdv = 0.0;
         if (!UPPER) {
             if (KIND == K_ITER && !SPLIT) {
@@ -209,7 +232,7 @@ __device__ __forceinline__ void run_chunk(uint8_t* __restrict__ st, int cnt_rt, 
             acc = fma(-v[k], d, acc);
         }
         if (UPPER) {
-            acc *= *(const double*)(R + 384 * W + 8 * lane);
+            acc *= *(const double*)(R + VROW * W + 8 * lane);
             if (SPLIT) {
                 sv[i * 32] = acc;                                  // z for the helper warp
                 if (GEN) out[pos] = acc;                           // GLOB entries read z from global
@@ -289,11 +312,11 @@ __device__ __forceinline__ void help_chunk(uint8_t* __restrict__ st, int recb, i
 // carries the chunk from one to the other (L: helper -> chain, U: chain -> helper).
 // cq: chunks consumed so far in the launch (mbarrier phase bookkeeping, identical in
 // both warps of a pair).
-template <int W, bool UPPER, int KIND, bool GEN, int ROLE>
+template <int W, bool UPPER, int KIND, bool GEN, int ROLE, int VB>
 __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, const WarpSmem& WS, unsigned& cq,
                                            int c, const PassOps& ops, double* out, double alpha, double& acc_dot,
                                            uint4* mb, unsigned ep) {
-    constexpr int RECB = 384 * W + (UPPER ? 256 : 0) + 16;
+    constexpr int RECB = (128 + 32 * VB) * W + (UPPER ? 256 : 0) + 16;
     constexpr bool SPLIT = ROLE != 0;
     const int lane = threadIdx.x & 31;
     const int64_t s0 = D.chain_step[c], s1 = D.chain_step[c + 1];
@@ -307,13 +330,17 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
         cnt = min(CC, nst - q * CC);
         glo = UPPER ? (s1 - (int64_t)q * CC - cnt) : (s0 + (int64_t)q * CC);
     };
-    auto stage_of = [&](int q) { return WS.stages + (size_t)((cq + q) % NST) * D.stage_bytes; };
-    auto issue = [&](int q) {               // lane 0 only
+    // ring slots: chunk q of the pass sits in slot (cq + q) mod NST with mbarrier phase
+    // ((cq + q) / NST) & 1; tracked incrementally (one division per pass, none per chunk)
+    auto stage_at = [&](unsigned slot) { return WS.stages + (size_t)slot * D.stage_bytes; };
+    auto next_slot = [&](unsigned& slot, unsigned& ph) {
+        if (++slot == (unsigned)NST) { slot = 0; ph ^= 1u; }
+    };
+    auto issue = [&](int q, unsigned slot) {               // lane 0 only
         int64_t glo;
         int cnt;
         chunk_range(q, glo, cnt);
-        const unsigned slot = (cq + q) % NST;
-        uint8_t* st = stage_of(q);
+        uint8_t* st = stage_at(slot);
         const unsigned rb = (unsigned)(cnt * RECB), vb = (unsigned)cnt * 256u;
         mbar_arrive_tx(&WS.full[slot], rb + vb * ops.nv);
         bulk_g2s(st, recs + (size_t)glo * RECB, rb, &WS.full[slot]);
@@ -321,16 +348,15 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
         for (int v = 0; v < ops.nv; ++v)
             bulk_g2s(vdst + (size_t)v * CC * 256, ops.v[v] + 32 * glo, vb, &WS.full[slot]);
     };
-    auto wait_bar = [&](uint64_t* bars, int q) -> bool {
-        const unsigned u = cq + q;
-        return warp_ok(mbar_wait(&bars[u % NST], (u / NST) & 1, E.sc));
+    auto wait_at = [&](uint64_t* bars, unsigned slot, unsigned ph) -> bool {
+        return warp_ok(mbar_wait(&bars[slot], ph, E.sc));
     };
     // ready flags of chunk q's cross-chain entries -> extq[q & 1] (one cp.async each)
-    auto prefetch_ext = [&](int q) {
+    auto prefetch_ext = [&](int q, unsigned slot) {
         int64_t glo;
         int cnt;
         chunk_range(q, glo, cnt);
-        const uint8_t* st = stage_of(q);
+        const uint8_t* st = stage_at(slot);
         uint4* qb = WS.extq + (size_t)(q & 1) * CC * 64;
         for (int i = 0; i < cnt; ++i) {
             const uint8_t* R = st + (size_t)i * RECB;
@@ -347,11 +373,11 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
     // of them together, until current: the chain then waits at most once per chunk (not
     // once per step), and the wait re-establishes a lag behind the producing chain of
     // about a chunk, so later prefetches find their values ready.
-    auto settle_ext = [&](int q) {
+    auto settle_ext = [&](int q, unsigned slot) {
         int64_t glo;
         int cnt;
         chunk_range(q, glo, cnt);
-        const uint8_t* st = stage_of(q);
+        const uint8_t* st = stage_at(slot);
         uint4* qb = WS.extq + (size_t)(q & 1) * CC * 64;
         const long long t0 = clock64();
         for (;;) {
@@ -364,14 +390,14 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
 #pragma unroll
                 for (int k = 0; k < W; ++k)
                     if ((tg[k] >> 29) == CT_EXT) {
-                        uint4* slot = qb + ((size_t)t * 2 + ((tg[k] >> 28) & 1)) * 32 + lane;
-                        uint4 f = *slot;
+                        uint4* slotp = qb + ((size_t)t * 2 + ((tg[k] >> 28) & 1)) * 32 + lane;
+                        uint4 f = *slotp;
                         if (f.y != ep || f.w != ep) {
                             asm volatile("ld.volatile.global.v4.u32 {%0, %1, %2, %3}, [%4];"
                                          : "=r"(f.x), "=r"(f.y), "=r"(f.z), "=r"(f.w)
                                          : "l"(mb + (tg[k] & 0x0fffffffu))
                                          : "memory");
-                            *slot = f;
+                            *slotp = f;
                             if (f.y != ep || f.w != ep) stale = true;
                         }
                     }
@@ -388,58 +414,72 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
     long long t_pass = SPCG_CHAIN_PROF ? clock64() : 0, t_wait = 0, t_ext = 0;
     GenCtx G{WS.hist, WS.extq, mb, E.sc, ep, GEN && (cfl & (UPPER ? CC_UHIST : CC_LHIST)) != 0};
     const bool rsrc_is_r = ops.v[0] == E.r;
-    if (ROLE != 2 && lane == 0)
-        for (int q = 0; q < min(NST, nch); ++q) issue(q);
+    const unsigned sl0 = cq % (unsigned)NST, ph0 = (cq / (unsigned)NST) & 1u;
+    if (ROLE != 2 && lane == 0) {
+        unsigned sl = sl0, ph = ph0;
+        for (int q = 0; q < min(NST, nch); ++q) {
+            issue(q, sl);
+            next_slot(sl, ph);
+        }
+    }
     if (use_ext && nch > 0) {
-        if (!wait_bar(WS.full, 0)) return;
-        prefetch_ext(0);
+        if (!wait_at(WS.full, sl0, ph0)) return;
+        prefetch_ext(0, sl0);
     }
     if (GEN && ROLE != 2) cpa_commit();
     double yprev = 0.0;
     double dot = acc_dot;
+    unsigned cs = sl0, cph = ph0;                        // slot / phase of chunk q
     for (int q = 0; q < nch; ++q) {
         int64_t glo;
         int cnt;
         chunk_range(q, glo, cnt);
-        uint8_t* st = stage_of(q);
+        unsigned ns_ = cs, nph = cph;                    // slot / phase of chunk q + 1
+        next_slot(ns_, nph);
+        uint8_t* st = stage_at(cs);
         if (ROLE == 2) {
             // helper: L before the chain (wait for the data), U after it (wait for the chain)
-            if (!wait_bar(UPPER ? WS.hand : WS.full, q)) return;
+            if (!wait_at(UPPER ? WS.hand : WS.full, cs, cph)) return;
             help_chunk<UPPER, KIND>(st, RECB, cnt, glo, ops.nv, rsrc_is_r, E.use_x0, out, E.r, E.xp, E.p, alpha, dot);
             __syncwarp();
             if (lane == 0) {
-                if (!UPPER) mbar_arrive(&WS.hand[(cq + q) % NST]);
-                else if (q + NST < nch) issue(q + NST);
+                if (!UPPER) mbar_arrive(&WS.hand[cs]);
+                else if (q + NST < nch) issue(q + NST, cs);
             }
+            cs = ns_;
+            cph = nph;
             continue;
         }
         long long t0 = SPCG_CHAIN_PROF ? clock64() : 0;
         if (GEN) {
             if (use_ext && q + 1 < nch) {
-                if (!wait_bar(WS.full, q + 1)) return;
-                prefetch_ext(q + 1);
+                if (!wait_at(WS.full, ns_, nph)) return;
+                prefetch_ext(q + 1, ns_);
             }
             cpa_commit();
             cpa_wait1();                                    // chunk q's flags landed
             G.qb = WS.extq + (size_t)(q & 1) * CC * 64;
-            if (use_ext) settle_ext(q);
+            if (use_ext) settle_ext(q, cs);
         }
         if (SPCG_CHAIN_PROF) { t_ext += clock64() - t0; t0 = clock64(); }
-        if (!wait_bar(SPLIT && !UPPER ? WS.hand : WS.full, q)) return;
+        if (!wait_at(SPLIT && !UPPER ? WS.hand : WS.full, cs, cph)) return;
         if (SPCG_CHAIN_PROF) t_wait += clock64() - t0;
         // full chunks of narrow records run fully unrolled (immediate offsets, loads of
         // later steps hoisted); wide records and the ragged last chunk take the loop
         if (W <= 4 && cnt == CC)
-            run_chunk<W, UPPER, KIND, GEN, SPLIT, (W <= 4 ? CC : 0)>(st, cnt, glo, q * CC, ops.nv, rsrc_is_r, E.use_x0,
-                                                                     out, E.r, E.xp, E.p, alpha, yprev, dot, G);
+            run_chunk<W, UPPER, KIND, GEN, SPLIT, (W <= 4 ? CC : 0), VB>(st, cnt, glo, q * CC, ops.nv, rsrc_is_r,
+                                                                         E.use_x0, out, E.r, E.xp, E.p, alpha, yprev,
+                                                                         dot, G);
         else
-            run_chunk<W, UPPER, KIND, GEN, SPLIT, 0>(st, cnt, glo, q * CC, ops.nv, rsrc_is_r, E.use_x0, out, E.r,
-                                                     E.xp, E.p, alpha, yprev, dot, G);
+            run_chunk<W, UPPER, KIND, GEN, SPLIT, 0, VB>(st, cnt, glo, q * CC, ops.nv, rsrc_is_r, E.use_x0, out, E.r,
+                                                         E.xp, E.p, alpha, yprev, dot, G);
         __syncwarp();
         if (lane == 0) {
-            if (SPLIT && UPPER) mbar_arrive(&WS.hand[(cq + q) % NST]);
-            if (refill && q + NST < nch) issue(q + NST);
+            if (SPLIT && UPPER) mbar_arrive(&WS.hand[cs]);
+            if (refill && q + NST < nch) issue(q + NST, cs);
         }
+        cs = ns_;
+        cph = nph;
     }
     if (GEN && ROLE != 2) cpa_wait0();
     cq += (unsigned)nch;
@@ -466,14 +506,22 @@ __device__ __forceinline__ void chain_pass_any(const DevChain& D, const PassEnv&
     const bool gen = UPPER ? (cfl & (CC_UHIST | CC_UEXT | CC_UGLOB | CC_UPUB)) != 0
                            : (cfl & (CC_LHIST | CC_LEXT | CC_LGLOB | CC_LPUB)) != 0;
     const int W = UPPER ? D.W_U : D.W_L;
-#define SPCG_CP(WW, GG, RR) chain_pass<WW, UPPER, KIND, GG, RR>(D, E, WS, cq, c, ops, out, alpha, acc_dot, mb, ep)
-#define SPCG_CPW(GG, RR)                          \
-    switch (W) {                                  \
-        case 1: SPCG_CP(1, GG, RR); break;        \
-        case 2: SPCG_CP(2, GG, RR); break;        \
-        case 4: SPCG_CP(4, GG, RR); break;        \
-        case 8: SPCG_CP(8, GG, RR); break;        \
-        default: SPCG_CP(16, GG, RR); break;      \
+#define SPCG_CP(WW, GG, RR, VV) chain_pass<WW, UPPER, KIND, GG, RR, VV>(D, E, WS, cq, c, ops, out, alpha, acc_dot, mb, ep)
+#define SPCG_CPW(GG, RR)                              \
+    if (D.vb == 4) {                                  \
+        switch (W) {                                  \
+            case 1: SPCG_CP(1, GG, RR, 4); break;     \
+            case 2: SPCG_CP(2, GG, RR, 4); break;     \
+            default: SPCG_CP(4, GG, RR, 4); break;    \
+        }                                             \
+    } else {                                          \
+        switch (W) {                                  \
+            case 1: SPCG_CP(1, GG, RR, 8); break;     \
+            case 2: SPCG_CP(2, GG, RR, 8); break;     \
+            case 4: SPCG_CP(4, GG, RR, 8); break;     \
+            case 8: SPCG_CP(8, GG, RR, 8); break;     \
+            default: SPCG_CP(16, GG, RR, 8); break;   \
+        }                                             \
     }
     if (role == 2) {      // the helper (the record width fixes the stage layout it reads)
         SPCG_CPW(false, 2)
