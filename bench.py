@@ -217,6 +217,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-host-setup", action="store_true", help="skip timing the host setup beside the GPU one")
     ap.add_argument("--no-f32", action="store_true", help="skip the fp32-factor (NEXT-2) leg of C4")
+    ap.add_argument("--no-multi-rhs", action="store_true", help="skip the multi-RHS (NEXT-4) leg of C4")
     ap.add_argument("--batch-count", type=int, default=64)
     ap.add_argument("--lanes", type=int, default=4,
                     help="C5: concurrent streams per GPU (each with SMs/lanes persistent CTAs)")
@@ -355,6 +356,32 @@ def main():
                "hbm_gbs_per_iter": fb * fk / (float(np.mean(fms)) * 1e-3) / 1e9, "status": inf["status"]}
         hf.close()
 
+    # NEXT-4: four right-hand sides of the same system in one launch (spcg_solve_multi):
+    # the matrix and factor streams are read once for all four
+    mrhs = None
+    if name == "C4" and not args.no_multi_rhs:
+        try:
+            Bh = np.stack([gen.rhs(A, seed=sd)[0] for sd in (99, 100, 101, 102)])
+            Bd = torch.from_numpy(Bh).to(f"cuda:{dev}")
+            h = handles["alg2"]
+            h.solve_multi(Bd, eps=EPS, kmax=KMAX)
+            mms, mk = [], None
+            for _ in range(max(1, min(args.steps, 3))):
+                flush.zero_()
+                _, infs = h.solve_multi(Bd, eps=EPS, kmax=KMAX)
+                mms.append(infs[0]["iter_phase_ms"])
+                mk = [i["iterations"] for i in infs]
+                assert all(i["status"] == 0 for i in infs), infs
+            mt = float(np.mean(mms))
+            mrhs = {"nrhs": 4, "ms": mt, "iterations": mk, "ms_per_rhs": mt / 4,
+                    "rhs_per_s": 4 / (mt * 1e-3), "single_rhs_ms": results["alg2"]["ms"],
+                    "throughput_vs_single": results["alg2"]["ms"] / (mt / 4),
+                    "ms_per_iter_all_rhs": mt / max(max(mk), 1),
+                    "note": "NEXT-4: 4 independent CGs, matrix/factor streams shared; right-hand sides "
+                            "b_j = A x_j with x_j from seeds 99..102"}
+        except Exception as e:        # a layout the multi-RHS kernel does not cover
+            mrhs = {"unavailable": str(e)[:200]}
+
     def mx(v):
         if ws == 1:
             return v
@@ -405,6 +432,7 @@ def main():
         "pcg": {"value": p_ms, "iterations": p["k"], "ms_per_iter": p_ms / max(p["k"], 1), "hbm_gbs_per_iter": p_gbs,
                 "algo_bytes_per_iter": p_bi, "levels": {"L": pi["levels_L"], "U": pi["levels_U"]}},
         "sweep": sweep or None,
+        "multi_rhs": mrhs,
         "fp32_factors": None if f32 is None else dict(f32, frac=f32["hbm_gbs_per_iter"] / peak,
                                                        note="NEXT-2: M = fl32(L) fl32(U) applied in fp64"),
         "spcg_vs_pcg": {"iter_phase_speedup": p_ms / s_ms,

@@ -242,7 +242,19 @@ spcg_status_t spcg_get_setup_info(spcg_handle_t h, spcg_setup_info_t* info);
 spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps, int64_t kmax,
                          uint32_t flags, spcg_solve_info_t* info);
 
-/* Asynchronous form of spcg_solve for running independent systems concurrently
+/* NEXT-4: nrhs right-hand sides of the same system, each an
+ * independent run of Algorithm 1 (own alpha, beta, stopping test; a converged one is
+ * frozen while the others continue), with the matrix and factor streams read once per
+ * group of up to 4.  B, X: device pointers, column-major n x nrhs
+ * (column j = right-hand side j), x0 = 0, flags must be 0.  info: array of nrhs entries
+ * (may be NULL); iter_phase_ms is the group's launch time.  Returns the worst status of
+ * the right-hand sides.  Requires the warp-chain executor whose chains need only
+ * shuffles (components / grid2d partitions without cross-chain terms), fp64 narrow
+ * records (W <= 4) and the TMA SpMV: otherwise SPCG_ERR_INVALID_ARG with the reason. */
+spcg_status_t spcg_solve_multi(spcg_handle_t h, const double* B, double* X, int32_t nrhs, double eps, int64_t kmax,
+                               uint32_t flags, spcg_solve_info_t* info);
+
+/* Asynchronous form of spcg_solve/* Asynchronous form of spcg_solve for running independent systems concurrently
  * (the C5 batch): enqueues Algorithm 1 on the handle's stream
  * and returns; b, x must be device pointers (SPCG_HOST_PTRS -> INVALID_ARG) and
  * stay valid until spcg_solve_wait(h, info) has returned, which synchronises

@@ -107,7 +107,8 @@ class SolveInfo(ctypes.Structure):
 EXPORTED = ["spcg_abi_version", "spcg_status_string", "spcg_last_error", "spcg_drop_params_default",
             "spcg_options_default", "spcg_setup", "spcg_get_setup_info", "spcg_solve", "spcg_apply_spmv",
             "spcg_apply_lower", "spcg_apply_upper", "spcg_apply_precond", "spcg_export", "spcg_destroy",
-            "spcg_calibrate", "spcg_solve_async", "spcg_solve_wait", "spcg_set_stream", "spcg_ll_stress"]
+            "spcg_calibrate", "spcg_solve_async", "spcg_solve_wait", "spcg_set_stream", "spcg_ll_stress",
+            "spcg_solve_multi"]
 
 
 def load(path: str | None = None):
@@ -153,6 +154,8 @@ def load(path: str | None = None):
     lib.spcg_set_stream.restype = I32
     lib.spcg_calibrate.argtypes = [I32, ctypes.POINTER(Calib)]
     lib.spcg_calibrate.restype = I32
+    lib.spcg_solve_multi.argtypes = [V, P, P, I32, D, I64, ctypes.c_uint32, ctypes.POINTER(SolveInfo)]
+    lib.spcg_solve_multi.restype = I32
     lib.spcg_ll_stress.argtypes = [I32, I32, I32, ctypes.POINTER(ctypes.c_uint64)]
     lib.spcg_ll_stress.restype = I32
     if lib.spcg_abi_version() != 3:
@@ -346,6 +349,21 @@ class SPCG:
         st = load().spcg_solve(self._h, b.data_ptr(), x.data_ptr(), float(eps), int(kmax), flags, ctypes.byref(info))
         _check(st, "spcg_solve")
         return x, self._solve_info(info)
+
+    def solve_multi(self, B, X=None, eps=1e-8, kmax=10000):
+        """spcg_solve_multi (NEXT-4): B is an (nrhs, n) float64 CUDA tensor, one right-hand
+        side per row (= the column-major n x nrhs block of the C ABI); returns (X, [info])."""
+        torch = _torch()
+        assert B.dtype == torch.float64 and B.is_cuda and B.is_contiguous() and B.dim() == 2 and B.shape[1] == self.n
+        nrhs = int(B.shape[0])
+        if X is None:
+            X = torch.empty_like(B)
+        self._order_after_current(B, X)
+        infos = (SolveInfo * nrhs)()
+        st = load().spcg_solve_multi(self._h, B.data_ptr(), X.data_ptr(), nrhs, float(eps), int(kmax), 0, infos)
+        if st < 0 and st != ERR_BREAKDOWN:
+            _check(st, "spcg_solve_multi")
+        return X, [self._solve_info(infos[j]) for j in range(nrhs)]
 
     def solve_async(self, b, x, eps=1e-8, kmax=10000):
         """spcg_solve_async: enqueue on the handle's stream (b, x device tensors kept alive by the caller)."""

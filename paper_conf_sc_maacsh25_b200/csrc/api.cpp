@@ -414,6 +414,49 @@ spcg_status_t spcg_get_setup_info(spcg_handle_t h, spcg_setup_info_t* info) {
     return SPCG_OK;
 }
 
+// NEXT-4: several right-hand sides of one system together
+spcg_status_t spcg_solve_multi(spcg_handle_t h, const double* B, double* X, int32_t nrhs, double eps, int64_t kmax,
+                               uint32_t flags, spcg_solve_info_t* info) {
+    if (!h || !B || !X || nrhs < 1 || kmax < 0 || !(eps >= 0.0)) {
+        set_error("bad solve_multi arguments");
+        return SPCG_ERR_INVALID_ARG;
+    }
+    if (flags != 0) { set_error("solve_multi: flags must be 0 (device pointers, x0 = 0)"); return SPCG_ERR_INVALID_ARG; }
+    if (kmax > SPCG_KMAX_LIMIT) { set_error("kmax > SPCG_KMAX_LIMIT"); return SPCG_ERR_INVALID_ARG; }
+    if (!h->dev) { set_error("host-only handle"); return SPCG_ERR_NO_DEVICE; }
+    try {
+        spcg_status_t worst = SPCG_OK;
+        for (int32_t g0 = 0; g0 < nrhs; g0 += 4) {            // groups of at most 4
+            const int m = std::min<int32_t>(4, nrhs - g0);
+            double out[16], ms = 0.0;
+            const double t0 = now_ms();
+            spcg_status_t st = spcg_dev_solve_multi(h->dev, B + (size_t)g0 * h->n, X + (size_t)g0 * h->n, m, eps, kmax,
+                                                    out, &ms);
+            if (st != SPCG_OK) return st;
+            for (int j = 0; j < m; ++j) {
+                if (!info) continue;
+                spcg_solve_info_t& I = info[g0 + j];
+                std::memset(&I, 0, sizeof I);
+                I.iterations = (int64_t)out[4 * j];
+                I.rnorm = std::sqrt(out[4 * j + 1]);
+                I.status = (spcg_status_t)out[4 * j + 2];
+                I.converged = I.status == SPCG_OK && eps > 0.0;
+                I.iter_phase_ms = ms;                         // one launch for the whole group
+                I.total_ms = now_ms() - t0;
+            }
+            for (int j = 0; j < m; ++j) {
+                const spcg_status_t sj = (spcg_status_t)out[4 * j + 2];
+                if (sj < 0 && (worst >= 0 || sj < worst)) worst = sj;
+                else if (sj == SPCG_NOT_CONVERGED && worst == SPCG_OK) worst = sj;
+            }
+        }
+        return worst;
+    } catch (...) {
+        set_error("unexpected exception in solve_multi");
+        return SPCG_ERR_INTERNAL;
+    }
+}
+
 spcg_status_t spcg_solve(spcg_handle_t h, const double* b, double* x, double eps, int64_t kmax,
                          uint32_t flags, spcg_solve_info_t* info) {
     if (!h || !b || !x || kmax < 0 || !(eps >= 0.0)) { set_error("bad solve arguments"); return SPCG_ERR_INVALID_ARG; }

@@ -85,7 +85,6 @@ struct DevChain {
     double* xp;                    // x in position order
     double* bp;                    // b (or the apply-mode input) in position order
     double* t1;                    // apply-mode temporary (position order)
-    double* p2;                    // second p buffer of the fused SpMV + direction update (wchain.cu)
 };
 
 struct Params {

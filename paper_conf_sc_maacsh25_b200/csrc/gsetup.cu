@@ -512,17 +512,75 @@ spcg_status_t levels(Ctx& C, const GCsr& M, const uint8_t* drop, bool lower, int
     return SPCG_OK;
 }
 
-spcg_status_t download(Ctx& C, const GCsr& M, spcg::Csr& out) {
+// Host <-> device copies of pageable std::vector data through two pinned bounce
+// buffers (a pageable cudaMemcpy runs at a few GB/s; this overlaps the host memcpy of
+// one chunk with the DMA of the other).
+constexpr size_t BOUNCE = 32u << 20;
+struct Bounce {
+    void* buf[2] = {nullptr, nullptr};
+    cudaEvent_t ev[2] = {nullptr, nullptr};
+    bool ok = false;
+    Bounce() {
+        ok = cudaMallocHost(&buf[0], BOUNCE) == cudaSuccess && cudaMallocHost(&buf[1], BOUNCE) == cudaSuccess &&
+             cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming) == cudaSuccess &&
+             cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming) == cudaSuccess;
+    }
+    ~Bounce() {
+        for (int k = 0; k < 2; ++k) {
+            if (ev[k]) cudaEventDestroy(ev[k]);
+            if (buf[k]) cudaFreeHost(buf[k]);
+        }
+    }
+};
+spcg_status_t h2d(Ctx& C, Bounce& B, void* dst, const void* src, size_t bytes) {
+    if (!B.ok) {
+        GCK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, C.s));
+        return SPCG_OK;
+    }
+    size_t off = 0;
+    for (int k = 0; off < bytes; k ^= 1) {
+        const size_t m = std::min(BOUNCE, bytes - off);
+        GCK(cudaEventSynchronize(B.ev[k]));                  // the DMA out of this buffer is done
+        std::memcpy(B.buf[k], (const char*)src + off, m);
+        GCK(cudaMemcpyAsync((char*)dst + off, B.buf[k], m, cudaMemcpyHostToDevice, C.s));
+        GCK(cudaEventRecord(B.ev[k], C.s));
+        off += m;
+    }
+    return SPCG_OK;
+}
+spcg_status_t d2h(Ctx& C, Bounce& B, void* dst, const void* src, size_t bytes) {
+    if (!B.ok) {
+        GCK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, C.s));
+        GCK(cudaStreamSynchronize(C.s));
+        return SPCG_OK;
+    }
+    // chunk j lands in buffer j & 1; it is drained while chunk j + 1 is in flight
+    const size_t nch = (bytes + BOUNCE - 1) / BOUNCE;
+    for (size_t j = 0; j < nch + 1; ++j) {
+        if (j < nch) {
+            const size_t off = j * BOUNCE, m = std::min(BOUNCE, bytes - off);
+            GCK(cudaMemcpyAsync(B.buf[j & 1], (const char*)src + off, m, cudaMemcpyDeviceToHost, C.s));
+            GCK(cudaEventRecord(B.ev[j & 1], C.s));
+        }
+        if (j > 0) {
+            const size_t i = j - 1, off = i * BOUNCE, m = std::min(BOUNCE, bytes - off);
+            GCK(cudaEventSynchronize(B.ev[i & 1]));
+            std::memcpy((char*)dst + off, B.buf[i & 1], m);
+        }
+    }
+    return SPCG_OK;
+}
+
+spcg_status_t download(Ctx& C, Bounce& B, const GCsr& M, spcg::Csr& out) {
     out.n = M.n;
     out.rp.resize(M.n + 1);
-    GCK(cudaMemcpyAsync(out.rp.data(), M.rp, 8 * (M.n + 1), cudaMemcpyDeviceToHost, C.s));
-    GCK(cudaStreamSynchronize(C.s));
+    spcg_status_t st;
+    if ((st = d2h(C, B, out.rp.data(), M.rp, 8 * (M.n + 1))) != SPCG_OK) return st;
     const int64_t nnz = out.rp[M.n];
     out.col.resize(nnz);
     out.val.resize(nnz);
-    GCK(cudaMemcpyAsync(out.col.data(), M.col, 4 * nnz, cudaMemcpyDeviceToHost, C.s));
-    GCK(cudaMemcpyAsync(out.val.data(), M.val, 8 * nnz, cudaMemcpyDeviceToHost, C.s));
-    return SPCG_OK;
+    if ((st = d2h(C, B, out.col.data(), M.col, 4 * nnz)) != SPCG_OK) return st;
+    return d2h(C, B, out.val.data(), M.val, 8 * nnz);
 }
 
 // compaction of A by a row predicate into a new device CSR
@@ -649,9 +707,11 @@ spcg_status_t gpu_setup_k0(const Csr& Ain, const spcg_drop_params_t& p, int devi
         set_error("gpu setup: device allocation failed");
         return SPCG_ERR_OOM;
     }
-    GCK(cudaMemcpyAsync(A.rp, Ain.rp.data(), 8 * (n + 1), cudaMemcpyHostToDevice, C.s));
-    GCK(cudaMemcpyAsync(A.col, Ain.col.data(), 4 * nnz, cudaMemcpyHostToDevice, C.s));
-    GCK(cudaMemcpyAsync(A.val, Ain.val.data(), 8 * nnz, cudaMemcpyHostToDevice, C.s));
+    Bounce B;
+    spcg_status_t st;
+    if ((st = h2d(C, B, A.rp, Ain.rp.data(), 8 * (n + 1))) != SPCG_OK) return st;
+    if ((st = h2d(C, B, A.col, Ain.col.data(), 4 * nnz)) != SPCG_OK) return st;
+    if ((st = h2d(C, B, A.val, Ain.val.data(), 8 * nnz)) != SPCG_OK) return st;
     {
         GErr e0{};
         e0.first_bad = ~0ull;
@@ -666,7 +726,7 @@ spcg_status_t gpu_setup_k0(const Csr& Ain, const spcg_drop_params_t& p, int devi
     unsigned long long counts[2];
     GCK(cudaMemcpyAsync(counts, C.cnt, 16, cudaMemcpyDeviceToHost, C.s));
     GErr he;
-    spcg_status_t st = check_err(C, he);
+    st = check_err(C, he);
     if (st != SPCG_OK) return st;
     if (he.first_bad != ~0ull) {
         const int64_t row = (int64_t)(he.first_bad >> 4);
@@ -769,13 +829,13 @@ spcg_status_t gpu_setup_k0(const Csr& Ain, const spcg_drop_params_t& p, int devi
     F.levL.resize(n);
     F.levU.resize(n);
     if ((st = levels(C, Ld, nullptr, true, lev, &F.wL)) != SPCG_OK) return st;
-    GCK(cudaMemcpyAsync(F.levL.data(), lev, 4 * n, cudaMemcpyDeviceToHost, C.s));
+    if ((st = d2h(C, B, F.levL.data(), lev, 4 * n)) != SPCG_OK) return st;
     if ((st = levels(C, Ud, nullptr, false, lev, &F.wU)) != SPCG_OK) return st;
-    GCK(cudaMemcpyAsync(F.levU.data(), lev, 4 * n, cudaMemcpyDeviceToHost, C.s));
+    if ((st = d2h(C, B, F.levU.data(), lev, 4 * n)) != SPCG_OK) return st;
     double t4 = now_ms();
-    if ((st = download(C, H, sp.Ahat)) != SPCG_OK) return st;
-    if ((st = download(C, Ld, F.L)) != SPCG_OK) return st;
-    if ((st = download(C, Ud, F.U)) != SPCG_OK) return st;
+    if ((st = download(C, B, H, sp.Ahat)) != SPCG_OK) return st;
+    if ((st = download(C, B, Ld, F.L)) != SPCG_OK) return st;
+    if ((st = download(C, B, Ud, F.U)) != SPCG_OK) return st;
     GCK(cudaStreamSynchronize(C.s));
     F.fill_level.assign(F.L.col.size() + F.U.col.size(), 0);
     double t5 = now_ms();

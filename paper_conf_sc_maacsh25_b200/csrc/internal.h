@@ -252,3 +252,5 @@ spcg_status_t spcg_dev_solve_end(spcg_device_t* d, spcg_solve_info_t* info, std:
 spcg_status_t spcg_dev_apply(spcg_device_t* d, int op, const double* in, double* out,
                              const double* aux, double* scalar_out);
 spcg_status_t spcg_dev_copy(spcg_device_t* d, void* dst, const void* src, size_t bytes, int kind);
+spcg_status_t spcg_dev_solve_multi(spcg_device_t* d, const double* B, double* X, int nrhs, double eps, int64_t kmax,
+                                   double* out_host, double* ms);

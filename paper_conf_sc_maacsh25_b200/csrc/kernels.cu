@@ -1463,6 +1463,7 @@ struct spcg_device_s {
     DevAllocator A{};                                 // caller's allocator hooks (or cudaMalloc)
     std::vector<std::pair<void*, size_t>> allocs;
     size_t mb_bytes = 0;                              // bytes of each ready-flag array (mbL, mbU)
+    int64_t glob_entries = 0;                         // wchain: own-chain dependencies read from global
     int64_t bytes = 0;
     unsigned epoch = 1;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -1478,6 +1479,11 @@ struct spcg_device_s {
     double* hist = nullptr;        // residual history buffer (grown on demand, reused)
     double* stage = nullptr;       // [2n] device copies of host b, x (SPCG_HOST_PTRS), allocated once
     long long hist_cap = 0;
+    // multi-RHS (NEXT-4, wchain_mrhs.cu): six position-major vectors of npos x mr_M, grown on demand
+    int mr_M = 0;
+    double* mr_vec[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    double* mr_part = nullptr;
+    double* mr_out = nullptr;
 };
 
 // debug: copy the heartbeat array while a kernel may still be running (own non-blocking stream)
@@ -1624,6 +1630,7 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         D.rec_L = CL.rec_L;
         D.rec_U = CL.rec_U;
         D.vb = CL.vb;
+        d->glob_entries = CL.glob_entries;
         D.nsteps = CL.nsteps;
         D.npos = nv;
         spcg::ChainSmemCfg cfg;
@@ -1671,7 +1678,6 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         AL(vb, P.CH.xp, double*);
         AL(vb, P.CH.bp, double*);
         AL(vb, P.CH.t1, double*);
-        AL(vb, P.CH.p2, double*);
     }
     AL(d->mb_bytes, P.mbL, uint4*);
     AL(d->mb_bytes, P.mbU, uint4*);
@@ -1781,6 +1787,85 @@ static spcg_status_t launch(spcg_device_t* d, Params& P) {
         CK(cudaLaunchKernel(pick_kernel(d->strategy), dim3(1), dim3(BLOCK), args, d->smem, d->stream));
     else
         CK(cudaLaunchCooperativeKernel(pick_kernel(d->strategy), dim3(d->parts), dim3(BLOCK), args, d->smem, d->stream));
+    return SPCG_OK;
+}
+
+void* spcg_wchain_mrhs_kernel_ptr(int M);     // wchain_mrhs.cu
+size_t spcg_mrhs_args_size();
+void spcg_mrhs_args_fill(void* dst, int nrhs, const double* B, double* X, double* const* vec, double* partials,
+                         double* out, int nst, unsigned stage_bytes, unsigned warp_bytes);
+
+// NEXT-4: nrhs (1..4) right-hand sides of the handle's system together.
+// B, X: device, column-major n x nrhs.  Requires the warp-chain executor with a chain
+// layout of pure shuffles (no ring / global / flag dependencies), narrow fp64 records and
+// the TMA SpMV.  Synchronous; out[m] = {k, ||r_k||^2, status}.
+spcg_status_t spcg_dev_solve_multi(spcg_device_t* d, const double* B, double* X, int nrhs, double eps, int64_t kmax,
+                                   double* out_host, double* ms) {
+    if (d->pending) { spcg::set_error("a solve is already in flight on this handle"); return SPCG_ERR_INVALID_ARG; }
+    const DevChain& D = d->P.CH;
+    if (d->strategy != ST_WCHAIN || D.any_ext || D.any_hist || d->glob_entries || D.W_L > 4 || D.W_U > 4 ||
+        D.vb != 8 || !(D.sp_nst >= 2 && D.WA >= 3 && D.WA <= 8)) {
+        spcg::set_error("multi-RHS solve needs the warp-chain executor with shuffle-only chains, narrow fp64 "
+                        "records and the TMA SpMV");
+        return SPCG_ERR_INVALID_ARG;
+    }
+    if (nrhs < 1 || nrhs > 4) { spcg::set_error("nrhs must be 1..4 per call"); return SPCG_ERR_INVALID_ARG; }
+    const int M = nrhs <= 2 ? 2 : 4;
+    CK(cudaSetDevice(d->device));
+    // stage sizing: CC steps of (record + operand slices of 256 M bytes), L needs 4 operands, U 2
+    const size_t C = spcg::SPCG_CHAIN_C;
+    const size_t stepL = (size_t)D.rec_L + 4 * 256 * (size_t)M, stepU = (size_t)D.rec_U + 2 * 256 * (size_t)M;
+    const size_t stage = (C * std::max(stepL, stepU) + 127) & ~(size_t)127;
+    int nst = (int)std::min<size_t>(16, spcg::SPCG_CHAIN_SMEM_LIMIT / ((size_t)D.per_cta * stage));
+    if (nst < 2) { spcg::set_error("multi-RHS stages do not fit shared memory"); return SPCG_ERR_INVALID_ARG; }
+    const size_t warp_bytes = stage * (size_t)nst;
+    const size_t smem = std::max((size_t)D.per_cta * warp_bytes, (size_t)8 * D.sp_nst * D.sp_stage_bytes);
+    if (M > d->mr_M) {
+        CK(cudaStreamSynchronize(d->stream));
+        for (auto& v : d->mr_vec)
+            if (v) { dev_free(d, v); v = nullptr; }
+        if (d->mr_part) { dev_free(d, d->mr_part); d->mr_part = nullptr; }
+        if (d->mr_out) { dev_free(d, d->mr_out); d->mr_out = nullptr; }
+        d->mr_M = 0;
+        void* p;
+        for (auto& v : d->mr_vec) {
+            spcg_status_t s = dev_malloc(d, sizeof(double) * (size_t)D.npos * M, &p);
+            if (s != SPCG_OK) return s;
+            v = (double*)p;
+        }
+        spcg_status_t s = dev_malloc(d, sizeof(double) * 4 * (size_t)M * d->parts, &p);
+        if (s != SPCG_OK) return s;
+        d->mr_part = (double*)p;
+        s = dev_malloc(d, sizeof(double) * 4 * (size_t)M, &p);
+        if (s != SPCG_OK) return s;
+        d->mr_out = (double*)p;
+        d->mr_M = M;
+    }
+    void* kfn = spcg_wchain_mrhs_kernel_ptr(M);
+    CK(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)spcg::SPCG_CHAIN_SMEM_LIMIT));
+    Params P = d->P;
+    P.mode = M_SOLVE;
+    P.eps = eps;
+    P.kmax = kmax;
+    std::vector<uint8_t> margs(spcg_mrhs_args_size());
+    spcg_mrhs_args_fill(margs.data(), nrhs, B, X, d->mr_vec, d->mr_part, d->mr_out, nst, (unsigned)stage,
+                        (unsigned)warp_bytes);
+    CK(cudaMemsetAsync(P.sc, 0, sizeof(Scal), d->stream));
+    void* args[] = {&P, margs.data()};
+    CK(cudaEventRecord(d->ev0, d->stream));
+    CK(cudaLaunchCooperativeKernel(kfn, dim3(d->parts), dim3(BLOCK), args, smem, d->stream));
+    CK(cudaEventRecord(d->ev1, d->stream));
+    CK(cudaMemcpyAsync(out_host, d->mr_out, sizeof(double) * 4 * M, cudaMemcpyDeviceToHost, d->stream));
+    Scal sc{};
+    CK(cudaMemcpyAsync(&sc, P.sc, sizeof(Scal), cudaMemcpyDeviceToHost, d->stream));
+    CK(cudaStreamSynchronize(d->stream));
+    float t = 0.f;
+    CK(cudaEventElapsedTime(&t, d->ev0, d->ev1));
+    *ms = t;
+    if (sc.status == SPCG_ERR_INTERNAL) {
+        spcg::set_error("multi-RHS solve aborted by its watchdog (internal)");
+        return SPCG_ERR_INTERNAL;
+    }
     return SPCG_OK;
 }
 
