@@ -480,13 +480,17 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_wchain_mrhs_kernel(Params P, MA
                 rr[m] = sums[M + m];
             }
         }
-        for (int64_t e = (int64_t)blockIdx.x * BLOCK + threadIdx.x; e < npos * M; e += stride) {
-            const int m = (int)(e % M);
-            double bm = beta[0];
-#pragma unroll
-            for (int j = 1; j < M; ++j)
-                if (m == j) bm = beta[j];
-            R.p[e] = fma(bm, R.p[e], __ldcg(R.z + e));
+        {   // p = z + beta p, 16-byte accesses (M is even: a pair never straddles two rows' RHS sets)
+            double2* p2 = (double2*)R.p;
+            const double2* z2 = (const double2*)R.z;
+            for (int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x; i < npos * M / 2; i += stride) {
+                double b0 = beta[0], b1 = beta[1];
+                if constexpr (M == 4) {
+                    if ((i & 1) != 0) { b0 = beta[2]; b1 = beta[3]; }
+                }
+                const double2 pv = p2[i], zv = __ldcg(z2 + i);
+                p2[i] = make_double2(fma(b0, pv.x, zv.x), fma(b1, pv.y, zv.y));
+            }
         }
         sync_tma(P.sc, gen);
         ++k;

@@ -1,5 +1,5 @@
 """C5 batch driver host logic: LPT plan and the multi-process gather (gloo,
-world_size 2, CPU), with host-only setups (device = -1)."""
+world_size 2 and 4, CPU), with host-only setups (device = -1)."""
 import os
 import socket
 
@@ -62,11 +62,12 @@ def _worker(rank, world, port, q):
     dist.destroy_process_group()
 
 
-def test_gather_two_ranks_gloo():
+@pytest.mark.parametrize("world", [2, 4])
+def test_gather_ranks_gloo(world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
     for p in procs:
         p.start()
     out = q.get(timeout=300)
