@@ -56,22 +56,20 @@ __device__ __forceinline__ void prof_phase(int idx, long long& t) {
 struct WarpSmem {
     uint64_t* full;        // [nst] mbarriers: TMA landed
     uint64_t* hand;        // [nst] mbarriers: handoff between the chain warp and its helper
-    uint64_t* freed;       // [nst] mbarriers: the chain warp has consumed the slot (the helper refills it)
     uint8_t* stages;       // nst x stage_bytes
     uint4* extq;           // [2][C][2][32] prefetched ready flags
     double* hist;          // [SPCG_CHAIN_HIST][32]
 };
 
-// per solver-warp slot: full[16] + hand[16] + freed[16] mbarriers, in static shared memory (the
+// per solver-warp slot: full[16] + hand[16] mbarriers, in static shared memory (the
 // dynamic area is reused by the SpMV's TMA stages between the triangular solves)
-__shared__ __align__(8) uint64_t s_chain_bar[NWARP][48];
+__shared__ __align__(8) uint64_t s_chain_bar[NWARP][32];
 
 __device__ __forceinline__ WarpSmem warp_smem(const DevChain& D, uint8_t* dyn, int sw) {
     WarpSmem W;
     uint8_t* base = dyn + (size_t)sw * D.warp_bytes;
     W.full = &s_chain_bar[sw][0];
     W.hand = &s_chain_bar[sw][16];
-    W.freed = &s_chain_bar[sw][32];
     W.stages = base;
     W.extq = (uint4*)(base + D.ext_off);
     W.hist = (double*)(base + D.hist_off);
@@ -309,9 +307,8 @@ __device__ __forceinline__ void help_chunk(uint8_t* __restrict__ st, int recb, i
 // One pass (L forward or U backward) of chain c: TMA-staged chunks of CC steps, NST
 // stages in flight; cross-chain ready flags of chunk q+1 prefetched (cp.async) while
 // chunk q runs.  ROLE 0: the chain warp alone; ROLE 1: the chain warp of a SPLIT pair;
-// ROLE 2: its helper warp.  In a pair, the chain warp issues the first NST chunks and the
-// helper every refill (U: after it read the stage; L: once the chain warp, the last
-// reader, marks the slot freed — so no TMA issue sits on the chain); hand[slot]
+// ROLE 2: its helper warp.  In a pair, the chain warp issues the first NST chunks, the
+// last reader of a stage refills it (L: the chain warp, U: the helper), and hand[slot]
 // carries the chunk from one to the other (L: helper -> chain, U: chain -> helper).
 // cq: chunks consumed so far in the launch (mbarrier phase bookkeeping, identical in
 // both warps of a pair).
@@ -412,6 +409,7 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
             }
         }
     };
+    const bool refill = ROLE == 0 || (ROLE == 1) == !UPPER;   // the last reader of a stage refills it
 
     long long t_pass = SPCG_CHAIN_PROF ? clock64() : 0, t_wait = 0, t_ext = 0;
     GenCtx G{WS.hist, WS.extq, mb, E.sc, ep, GEN && (cfl & (UPPER ? CC_UHIST : CC_LHIST)) != 0};
@@ -432,7 +430,6 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
     double yprev = 0.0;
     double dot = acc_dot;
     unsigned cs = sl0, cph = ph0;                        // slot / phase of chunk q
-    unsigned ps = 0, pph = 0;                            // helper: slot / phase of chunk q - 1
     for (int q = 0; q < nch; ++q) {
         int64_t glo;
         int cnt;
@@ -449,14 +446,6 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
                 if (!UPPER) mbar_arrive(&WS.hand[cs]);
                 else if (q + NST < nch) issue(q + NST, cs);
             }
-            // L: the helper also refills, one chunk behind — chunk q-1+NST goes into the slot
-            // of chunk q-1 once the chain warp has freed it (the TMA issue stays off the chain)
-            if (!UPPER && q >= 1 && q - 1 + NST < nch) {
-                if (!wait_at(WS.freed, ps, pph)) return;
-                if (lane == 0) issue(q - 1 + NST, ps);
-            }
-            ps = cs;
-            pph = cph;
             cs = ns_;
             cph = nph;
             continue;
@@ -486,13 +475,8 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
                                                          E.xp, E.p, alpha, yprev, dot, G);
         __syncwarp();
         if (lane == 0) {
-            if (SPLIT) {
-                // freed[] completes once per chunk in every pass (its phase follows cq); only
-                // the L helper waits on it
-                mbar_arrive(&WS.freed[cs]);
-                if (UPPER) mbar_arrive(&WS.hand[cs]);
-            }
-            if (ROLE == 0 && q + NST < nch) issue(q + NST, cs);
+            if (SPLIT && UPPER) mbar_arrive(&WS.hand[cs]);
+            if (refill && q + NST < nch) issue(q + NST, cs);
         }
         cs = ns_;
         cph = nph;
@@ -808,7 +792,6 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_wchain_kernel(Params P) {
             for (int s = 0; s < D.nst; ++s) {
                 mbar_init(&W.full[s], 1);
                 mbar_init(&W.hand[s], 1);
-                mbar_init(&W.freed[s], 1);
             }
         }
         for (int i = 0; i < NWARP * 4; ++i) mbar_init(&spbar[i], 1);
