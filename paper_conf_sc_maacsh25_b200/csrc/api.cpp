@@ -30,8 +30,8 @@ struct spcg_handle_s {
     std::vector<double> rhist;
 };
 
-template <class T>
-static spcg_status_t put(const std::vector<T>& v, void* buf, size_t* bytes) {
+template <class T, class Al>
+static spcg_status_t put(const std::vector<T, Al>& v, void* buf, size_t* bytes) {
     size_t need = v.size() * sizeof(T);
     if (!buf) { *bytes = need; return SPCG_OK; }
     if (*bytes < need) { set_error("export buffer too small"); return SPCG_ERR_INVALID_ARG; }

@@ -188,7 +188,7 @@ bool part_grid2d(const Factors& F, ChainPart& out) {
 }
 
 template <class T>
-void put(std::vector<uint8_t>& b, size_t off, T v) { std::memcpy(b.data() + off, &v, sizeof(T)); }
+void put(fast_vector<uint8_t>& b, size_t off, T v) { std::memcpy(b.data() + off, &v, sizeof(T)); }
 
 }  // namespace
 
@@ -236,22 +236,40 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, bool 
     for (int32_t c = 0; c < CP.nchains; ++c)
         std::stable_sort(rows.begin() + cstart[c], rows.begin() + cstart[c + 1],
                          [&](int32_t x, int32_t y) { return key(x) < key(y); });
-    for (int32_t c = 0; c < CP.nchains; ++c) {
-        if (remap[c] < 0) continue;
+    // steps of each chain (parallel over chains), their prefix, then the rows' steps/lanes
+    std::vector<int64_t> csteps(CP.nchains, 0);
+    auto walk = [&](int32_t c, int64_t g0, bool assign) {
         auto b = rows.begin() + cstart[c], e = rows.begin() + cstart[c + 1];
-        out.chain_step[remap[c]] = g;
+        int64_t gg = g0;
         for (auto it = b; it != e;) {
             auto jt = it;
             int lane = 0;
             while (jt != e && key(*jt) == key(*it) && lane < 32) {
-                step_of[*jt] = g;
-                lane_of[*jt] = lane++;
+                if (assign) {
+                    step_of[*jt] = gg;
+                    lane_of[*jt] = lane;
+                }
+                ++lane;
                 ++jt;
             }
-            ++g;
+            ++gg;
             it = jt;
         }
+        return gg - g0;
+    };
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int32_t c = 0; c < CP.nchains; ++c)
+        if (remap[c] >= 0) csteps[c] = walk(c, 0, false);
+    std::vector<int64_t> cfirst(CP.nchains, 0);
+    for (int32_t c = 0; c < CP.nchains; ++c) {
+        if (remap[c] < 0) continue;
+        out.chain_step[remap[c]] = g;
+        cfirst[c] = g;
+        g += csteps[c];
     }
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int32_t c = 0; c < CP.nchains; ++c)
+        if (remap[c] >= 0) walk(c, cfirst[c], true);
     out.chain_step[nch] = g;
     out.nsteps = g;
     const int64_t npos = 32 * g;
@@ -260,9 +278,11 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, bool 
         return false;
     }
     std::vector<int32_t> chain(n);
+#pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < n; ++i) chain[i] = remap[CP.chain_of[i]];
     out.perm.assign(npos, -1);
     out.iperm.assign(n, 0);
+#pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < n; ++i) {
         const int64_t p = 32 * step_of[i] + lane_of[i];
         out.perm[p] = (int32_t)i;
@@ -278,8 +298,13 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, bool 
     const int vrow = 128 + 32 * out.vb;   // bytes per entry column of a record: tags + values
     out.rec_L = vrow * out.W_L + 16;
     out.rec_U = vrow * out.W_U + 256 + 16;
-    out.recL.assign((size_t)g * out.rec_L, 0);
-    out.recU.assign((size_t)g * out.rec_U, 0);
+    out.recL.resize((size_t)g * out.rec_L);         // uninitialised: zeroed below by step, in parallel
+    out.recU.resize((size_t)g * out.rec_U);
+#pragma omp parallel for schedule(static)
+    for (int64_t s = 0; s < g; ++s) {
+        std::memset(out.recL.data() + (size_t)s * out.rec_L, 0, out.rec_L);
+        std::memset(out.recU.data() + (size_t)s * out.rec_U, 0, out.rec_U);
+    }
     out.chain_flags.assign(nch, 0u);
 
     // records: for each row, its dependencies in CSR order (the order of the definition)
@@ -287,7 +312,7 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, bool 
         const Csr& M = upper ? F.U : F.L;
         const int W = upper ? out.W_U : out.W_L;
         const int rb = upper ? out.rec_U : out.rec_L;
-        std::vector<uint8_t>& R = upper ? out.recU : out.recL;
+        fast_vector<uint8_t>& R = upper ? out.recU : out.recL;
         const size_t trailer = (size_t)vrow * W + (upper ? 256 : 0);
         int64_t n_prev = 0, n_hist = 0, n_glob = 0, n_ext = 0;
         bool bad = false;
@@ -382,8 +407,8 @@ bool build_chain_layout(const Csr& A, const Factors& F, int target_chains, bool 
     out.WA = (int32_t)WA;
     S.eoff.assign(g + 1, 0);
     for (int64_t s = 0; s < g; ++s) S.eoff[s + 1] = S.eoff[s] + WA;
-    S.col.assign(S.eoff[g] * 32, 0);
-    S.val.assign(S.eoff[g] * 32, 0.0);
+    S.col.resize(S.eoff[g] * 32);                    // every element is written below
+    S.val.resize(S.eoff[g] * 32);
 #pragma omp parallel for schedule(static)
     for (int64_t s = 0; s < g; ++s)
         for (int l = 0; l < 32; ++l) {

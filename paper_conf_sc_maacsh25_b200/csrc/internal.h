@@ -2,6 +2,8 @@
 // Not part of the ABI (include/spcg.h is).  No oracle code or header is used here.
 #pragma once
 #include <cstdint>
+#include <memory>
+#include <utility>
 #include <string>
 #include <vector>
 
@@ -10,6 +12,23 @@
 struct DevAllocator;               // spcg_options_t allocator hooks (defined below)
 
 namespace spcg {
+
+// Allocator whose value-construction is a no-op: the large layout arrays are filled in
+// parallel (first touch by the filling threads) instead of zeroed by one thread first.
+template <class T>
+struct NoInit : std::allocator<T> {
+    template <class U>
+    struct rebind { using other = NoInit<U>; };
+    NoInit() = default;
+    template <class U>
+    NoInit(const NoInit<U>&) {}
+    template <class U>
+    void construct(U* p) { ::new ((void*)p) U; }
+    template <class U, class... A>
+    void construct(U* p, A&&... a) { ::new ((void*)p) U(std::forward<A>(a)...); }
+};
+template <class T>
+using fast_vector = std::vector<T, NoInit<T>>;
 
 struct Csr {                       // host CSR, int64 row pointers
     int64_t n = 0;
@@ -104,8 +123,8 @@ constexpr int SPCG_RES_WARPS = 8;      // warps of the resident CTA (slice s -> 
 struct SpmvLayout {                // SELL-32 of the original A, natural row order
     int32_t nslices = 0;
     std::vector<int64_t> eoff;
-    std::vector<int32_t> col;
-    std::vector<double> val;
+    fast_vector<int32_t> col;      // every element written by the builder (no zero pass)
+    fast_vector<double> val;
 };
 
 // Chunked executor stream.  Per part (CTA) one byte stream of
@@ -178,7 +197,7 @@ struct ChainLayout {
     std::vector<uint32_t> chain_flags;    // [nchains] CC_*
     std::vector<int32_t> perm;            // [npos] row at each position (-1 padding)
     std::vector<int32_t> iperm;           // [n] position of each row
-    std::vector<uint8_t> recL, recU;      // nsteps records each
+    fast_vector<uint8_t> recL, recU;      // nsteps records each (zeroed in parallel by the builder)
     SpmvLayout A;                         // SELL-32 of A over positions (slice = step), uniform width WA
     int32_t WA = 0;
     std::string partition;                // components / grid2d / grid3d

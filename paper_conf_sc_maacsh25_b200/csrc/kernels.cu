@@ -1527,8 +1527,8 @@ static void dev_free(spcg_device_t* d, void* p) {
         }
 }
 
-template <class T>
-static spcg_status_t upload(spcg_device_t* d, const std::vector<T>& v, const T** out) {
+template <class T, class Al>
+static spcg_status_t upload(spcg_device_t* d, const std::vector<T, Al>& v, const T** out) {
     void* p = nullptr;
     spcg_status_t s = dev_malloc(d, v.size() * sizeof(T), &p);
     if (s != SPCG_OK) return s;

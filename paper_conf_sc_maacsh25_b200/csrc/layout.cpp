@@ -38,7 +38,7 @@ void build_spmv_layout(const Csr& A, SpmvLayout& out) {
         for (int64_t r = 32LL * s; r < std::min<int64_t>(n, 32LL * s + 32); ++r) w = std::max(w, A.rp[r + 1] - A.rp[r]);
         out.eoff[s + 1] = out.eoff[s] + w;
     }
-    out.col.assign(out.eoff[ns] * 32, 0);
+    out.col.assign(out.eoff[ns] * 32, 0);          // (sequential builder: keeps the zero fill)
     out.val.assign(out.eoff[ns] * 32, 0.0);
     for (int32_t s = 0; s < ns; ++s)
         for (int l = 0; l < 32; ++l) {

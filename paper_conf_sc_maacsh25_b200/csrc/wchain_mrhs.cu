@@ -480,16 +480,29 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_wchain_mrhs_kernel(Params P, MA
                 rr[m] = sums[M + m];
             }
         }
-        {   // p = z + beta p, 16-byte accesses (M is even: a pair never straddles two rows' RHS sets)
-            double2* p2 = (double2*)R.p;
-            const double2* z2 = (const double2*)R.z;
-            for (int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x; i < npos * M / 2; i += stride) {
-                double b0 = beta[0], b1 = beta[1];
-                if constexpr (M == 4) {
-                    if ((i & 1) != 0) { b0 = beta[2]; b1 = beta[3]; }
-                }
-                const double2 pv = p2[i], zv = __ldcg(z2 + i);
-                p2[i] = make_double2(fma(b0, pv.x, zv.x), fma(b1, pv.y, zv.y));
+        {   // p = z + beta p, 16-byte accesses (M is even: a pair never straddles two rows' RHS
+            // sets), four of them in flight per thread before the first store
+            double2* __restrict__ p2 = (double2*)R.p;
+            const double2* __restrict__ z2 = (const double2*)R.z;
+            const int64_t n2 = npos * M / 2;
+            for (int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x; i < n2; i += 4 * stride) {
+                double2 pv[4], zv[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+                    if (i + u * stride < n2) {
+                        pv[u] = p2[i + u * stride];
+                        zv[u] = __ldcg(z2 + i + u * stride);
+                    }
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+                    if (i + u * stride < n2) {
+                        const int64_t j = i + u * stride;
+                        double b0 = beta[0], b1 = beta[1];
+                        if constexpr (M == 4) {
+                            if ((j & 1) != 0) { b0 = beta[2]; b1 = beta[3]; }
+                        }
+                        p2[j] = make_double2(fma(b0, pv[u].x, zv[u].x), fma(b1, pv[u].y, zv[u].y));
+                    }
             }
         }
         sync_tma(P.sc, gen);
