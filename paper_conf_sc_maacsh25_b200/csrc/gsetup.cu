@@ -134,7 +134,11 @@ __global__ void k_validate(int64_t n, const int64_t* __restrict__ rp, const int3
 __global__ void k_levels(int64_t n, const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
                          const uint8_t* __restrict__ drop, int lower, int* lev, unsigned long long* counter,
                          GErr* err) {
-    const int lane = threadIdx.x & 31;
+    // A dependency inside the warp's own 32 rows (lane l on lane l-1: every natural-order
+    // grid) is resolved through shared memory in rounds of __syncwarp, not by re-polling
+    // global memory: a chain of 32 lanes costs 32 short rounds, not 32 L2 round trips.
+    __shared__ int slv[GB / 32][32];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     int mymax = -1;
     for (;;) {
         unsigned long long base = 0;
@@ -143,24 +147,51 @@ __global__ void k_levels(int64_t n, const int64_t* __restrict__ rp, const int32_
         if ((int64_t)base >= n) break;
         const int64_t t = (int64_t)base + lane;
         const int64_t i = lower ? t : n - 1 - t;
-        bool done = t >= n;
+        // rows of this chunk: lower [base, base + 32), upper [n - base - 32, n - base)
+        const int64_t lo = lower ? (int64_t)base : n - (int64_t)base - 32, hi = lo + 31;
+        bool done = t >= n, ext_ok = done;
+        int ext_max = -1, lvl = -1;
+        slv[wib][lane] = -1;
+        __syncwarp();
         const long long t0 = clock64();
         for (;;) {
-            if (!done) {
-                int m = -1;
+            if (!ext_ok) {
                 bool ok = true;
+                int m = -1;
                 for (int64_t q = rp[i]; q < rp[i + 1]; ++q) {
                     const int64_t j = col[q];
-                    if ((lower ? j >= i : j <= i) || (drop && drop[q])) continue;
+                    if ((lower ? j >= i : j <= i) || (drop && drop[q]) || (j >= lo && j <= hi)) continue;
                     const int v = ld_vol(lev + j);
                     if (v < 0) { ok = false; break; }
                     m = max(m, v);
                 }
-                if (ok) {
-                    st_vol(lev + i, m + 1);
-                    mymax = max(mymax, m + 1);
-                    done = true;
+                if (ok) { ext_ok = true; ext_max = m; }
+            }
+            // internal rounds: a lane whose external part is known finishes once its
+            // dependencies inside the chunk have (they are earlier lanes)
+            for (int r = 0; r < 32; ++r) {
+                bool progressed = false;
+                if (ext_ok && !done) {
+                    int m = ext_max;
+                    bool ok = true;
+                    for (int64_t q = rp[i]; q < rp[i + 1]; ++q) {
+                        const int64_t j = col[q];
+                        if ((lower ? j >= i : j <= i) || (drop && drop[q]) || j < lo || j > hi) continue;
+                        const int v = *(volatile int*)&slv[wib][lower ? (int)(j - lo) : (int)(hi - j)];
+                        if (v < 0) { ok = false; break; }
+                        m = max(m, v);
+                    }
+                    if (ok) {
+                        lvl = m + 1;
+                        slv[wib][lane] = lvl;
+                        st_vol(lev + i, lvl);
+                        mymax = max(mymax, lvl);
+                        done = true;
+                        progressed = true;
+                    }
                 }
+                __syncwarp();
+                if (!__any_sync(0xffffffffu, progressed)) break;
             }
             if (__all_sync(0xffffffffu, done)) break;
             if (__any_sync(0xffffffffu, clock64() - t0 > G_SPIN_TIMEOUT || ld_vol(&err->abort) != 0)) {
@@ -168,6 +199,7 @@ __global__ void k_levels(int64_t n, const int64_t* __restrict__ rp, const int32_
                 return;
             }
         }
+        __syncwarp();
     }
     for (int o = 16; o; o >>= 1) mymax = max(mymax, __shfl_xor_sync(0xffffffffu, mymax, o));
     if (lane == 0) atomicMax(&err->max_level, mymax);
@@ -373,45 +405,70 @@ __global__ void k_compact(int64_t n, const int64_t* __restrict__ rp, const int32
 __global__ void k_ilu0(int64_t n, const int64_t* __restrict__ lrp, const int32_t* __restrict__ lcol,
                        double* lval, const int64_t* __restrict__ urp, const int32_t* __restrict__ ucol, double* uval,
                        int* done, unsigned long long* counter, GErr* err) {
-    const int lane = threadIdx.x & 31;
+    // rows of an L dependency inside the warp's 32-row chunk are waited for through a
+    // shared-memory flag and __syncwarp (which orders the warp's global stores before the
+    // dependent lane's loads), the rest through the global acquire / release flags
+    __shared__ int sdone[GB / 32][32];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     for (;;) {
         unsigned long long base = 0;
         if (lane == 0) base = atomicAdd(counter, 32ull);
         base = __shfl_sync(0xffffffffu, base, 0);
         if ((int64_t)base >= n) break;
         const int64_t i = (int64_t)base + lane;
-        bool fin = i >= n;
+        const int64_t lo = (int64_t)base;
+        bool fin = i >= n, ext_ok = fin;
+        sdone[wib][lane] = fin ? 1 : 0;
+        __syncwarp();
         const long long t0 = clock64();
         for (;;) {
-            if (!fin) {
+            if (!ext_ok) {
                 bool ok = true;
-                for (int64_t q = lrp[i]; q < lrp[i + 1]; ++q)
-                    if (ld_acq(done + lcol[q]) == 0) { ok = false; break; }
-                if (ok) {
-                    const int64_t l0 = lrp[i], l1 = lrp[i + 1], u0i = urp[i], u1i = urp[i + 1];
-                    for (int64_t q = l0; q < l1; ++q) {
+                for (int64_t q = lrp[i]; q < lrp[i + 1]; ++q) {
+                    const int64_t k = lcol[q];
+                    if (k >= lo) continue;                             // inside the chunk
+                    if (ld_acq(done + k) == 0) { ok = false; break; }
+                }
+                ext_ok = ok;
+            }
+            for (int r = 0; r < 32; ++r) {
+                bool progressed = false;
+                if (ext_ok && !fin) {
+                    bool ok = true;
+                    for (int64_t q = lrp[i]; q < lrp[i + 1]; ++q) {
                         const int64_t k = lcol[q];
-                        const int64_t uk0 = urp[k], uk1 = urp[k + 1];
-                        const double lik = __ddiv_rn(lval[q], __ldcg(uval + uk0));
-                        lval[q] = lik;
-                        int64_t pl = q + 1, pu = u0i;
-                        for (int64_t r = uk0 + 1; r < uk1; ++r) {
-                            const int32_t j = __ldcg(ucol + r);
-                            const double ukj = __ldcg(uval + r);
-                            if (j < i) {
-                                while (pl < l1 && lcol[pl] < j) ++pl;
-                                if (pl < l1 && lcol[pl] == j) lval[pl] = __dsub_rn(lval[pl], __dmul_rn(lik, ukj));
-                            } else {
-                                while (pu < u1i && ucol[pu] < j) ++pu;
-                                if (pu < u1i && ucol[pu] == j) uval[pu] = __dsub_rn(uval[pu], __dmul_rn(lik, ukj));
+                        if (k >= lo && *(volatile int*)&sdone[wib][(int)(k - lo)] == 0) { ok = false; break; }
+                    }
+                    if (ok) {
+                        const int64_t l0 = lrp[i], l1 = lrp[i + 1], u0i = urp[i], u1i = urp[i + 1];
+                        for (int64_t q = l0; q < l1; ++q) {
+                            const int64_t k = lcol[q];
+                            const int64_t uk0 = urp[k], uk1 = urp[k + 1];
+                            const double lik = __ddiv_rn(lval[q], __ldcg(uval + uk0));
+                            lval[q] = lik;
+                            int64_t pl = q + 1, pu = u0i;
+                            for (int64_t rr = uk0 + 1; rr < uk1; ++rr) {
+                                const int32_t j = __ldcg(ucol + rr);
+                                const double ukj = __ldcg(uval + rr);
+                                if (j < i) {
+                                    while (pl < l1 && lcol[pl] < j) ++pl;
+                                    if (pl < l1 && lcol[pl] == j) lval[pl] = __dsub_rn(lval[pl], __dmul_rn(lik, ukj));
+                                } else {
+                                    while (pu < u1i && ucol[pu] < j) ++pu;
+                                    if (pu < u1i && ucol[pu] == j) uval[pu] = __dsub_rn(uval[pu], __dmul_rn(lik, ukj));
+                                }
                             }
                         }
+                        const double d = uval[u0i];
+                        if (d == 0.0 || !isfinite(d)) atomicMin(&err->bad_pivot, (unsigned long long)i);
+                        st_rel(done + i, 1);
+                        sdone[wib][lane] = 1;
+                        fin = true;
+                        progressed = true;
                     }
-                    const double d = uval[u0i];
-                    if (d == 0.0 || !isfinite(d)) atomicMin(&err->bad_pivot, (unsigned long long)i);
-                    st_rel(done + i, 1);
-                    fin = true;
                 }
+                __syncwarp();
+                if (!__any_sync(0xffffffffu, progressed)) break;
             }
             if (__all_sync(0xffffffffu, fin)) break;
             if (__any_sync(0xffffffffu, clock64() - t0 > G_SPIN_TIMEOUT || ld_vol(&err->abort) != 0)) {
@@ -419,6 +476,7 @@ __global__ void k_ilu0(int64_t n, const int64_t* __restrict__ lrp, const int32_t
                 return;
             }
         }
+        __syncwarp();
     }
 }
 

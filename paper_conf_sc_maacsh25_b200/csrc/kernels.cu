@@ -1481,7 +1481,7 @@ struct spcg_device_s {
     long long hist_cap = 0;
     // multi-RHS (NEXT-4, wchain_mrhs.cu): six position-major vectors of npos x mr_M, grown on demand
     int mr_M = 0;
-    double* mr_vec[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    double* mr_vec[12] = {};       // [vector r, w, p, z, y, xp][half]
     double* mr_part = nullptr;
     double* mr_out = nullptr;
 };
@@ -1811,15 +1811,18 @@ spcg_status_t spcg_dev_solve_multi(spcg_device_t* d, const double* B, double* X,
     }
     if (nrhs < 1 || nrhs > 4) { spcg::set_error("nrhs must be 1..4 per call"); return SPCG_ERR_INVALID_ARG; }
     const int M = nrhs <= 2 ? 2 : 4;
+    const int H = M / 2;                  // right-hand-side halves of two: one chain warp each
+    if (H * D.per_cta > NWARP) { spcg::set_error("multi-RHS: too many chains per CTA"); return SPCG_ERR_INVALID_ARG; }
     CK(cudaSetDevice(d->device));
-    // stage sizing: CC steps of (record + operand slices of 256 M bytes), L needs 4 operands, U 2
+    // stage sizing per chain warp: CC steps of (record + operand slices of 2 x 256 bytes), L
+    // needs 4 operands, U 2
     const size_t C = spcg::SPCG_CHAIN_C;
-    const size_t stepL = (size_t)D.rec_L + 4 * 256 * (size_t)M, stepU = (size_t)D.rec_U + 2 * 256 * (size_t)M;
+    const size_t stepL = (size_t)D.rec_L + 4 * 512, stepU = (size_t)D.rec_U + 2 * 512;
     const size_t stage = (C * std::max(stepL, stepU) + 127) & ~(size_t)127;
-    int nst = (int)std::min<size_t>(16, spcg::SPCG_CHAIN_SMEM_LIMIT / ((size_t)D.per_cta * stage));
+    int nst = (int)std::min<size_t>(16, spcg::SPCG_CHAIN_SMEM_LIMIT / ((size_t)H * D.per_cta * stage));
     if (nst < 2) { spcg::set_error("multi-RHS stages do not fit shared memory"); return SPCG_ERR_INVALID_ARG; }
     const size_t warp_bytes = stage * (size_t)nst;
-    const size_t smem = std::max((size_t)D.per_cta * warp_bytes, (size_t)8 * D.sp_nst * D.sp_stage_bytes);
+    const size_t smem = std::max((size_t)H * D.per_cta * warp_bytes, (size_t)8 * D.sp_nst * D.sp_stage_bytes);
     if (M > d->mr_M) {
         CK(cudaStreamSynchronize(d->stream));
         for (auto& v : d->mr_vec)
@@ -1828,8 +1831,10 @@ spcg_status_t spcg_dev_solve_multi(spcg_device_t* d, const double* B, double* X,
         if (d->mr_out) { dev_free(d, d->mr_out); d->mr_out = nullptr; }
         d->mr_M = 0;
         void* p;
-        for (auto& v : d->mr_vec) {
-            spcg_status_t s = dev_malloc(d, sizeof(double) * (size_t)D.npos * M, &p);
+        for (int k = 0; k < 12; ++k) {        // [vector][half]: r, w, p, z, y, xp
+            double*& v = d->mr_vec[k];
+            if ((k & 1) >= H) continue;
+            spcg_status_t s = dev_malloc(d, sizeof(double) * (size_t)D.npos * 2, &p);
             if (s != SPCG_OK) return s;
             v = (double*)p;
         }

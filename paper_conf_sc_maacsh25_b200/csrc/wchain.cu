@@ -678,17 +678,20 @@ __device__ void chain_spmv_tma(const DevChain& D, const DevA& A, uint8_t* dyn, u
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t ns = A.nslices;
     const int64_t NW = (int64_t)gridDim.x * NWARP, gw = (int64_t)blockIdx.x * NWARP + warp;
-    const int64_t a = gw * ns / NW, b = (gw + 1) * ns / NW;
+    // groups of G slices dealt round-robin over the grid's warps (group gi = j NW + gw): the
+    // positions of weak-coupling fragments cluster at the end of the layout, and contiguous
+    // ranges left the warps that got them (far gathers) the last to reach the barrier
+    const int64_t ngr = (ns + G - 1) / G;
     const int NS = D.sp_nst, WA = D.WA;
     uint8_t* ring = dyn + (size_t)warp * NS * D.sp_stage_bytes;
     uint64_t* bar = bars + warp * 4;
-    const int nst = (int)((b - a + G - 1) / G);
+    const int nst = (int)(gw < ngr ? (ngr - gw + NW - 1) / NW : 0);
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic reads of this smem done
     __syncwarp();
     auto issue = [&](int j) {
         const int slot = (spq + j) % NS;
-        const int64_t s = a + (int64_t)j * G;
-        const int g = (int)(b - s < (int64_t)G ? b - s : (int64_t)G);
+        const int64_t s = ((int64_t)j * NW + gw) * G;
+        const int g = (int)(ns - s < (int64_t)G ? ns - s : (int64_t)G);
         const unsigned cb = (unsigned)(g * WA * 128), vb = (unsigned)(g * WA * 256);
         uint8_t* st = ring + (size_t)slot * D.sp_stage_bytes;
         mbar_arrive_tx(&bar[slot], cb + vb);
@@ -706,8 +709,8 @@ __device__ void chain_spmv_tma(const DevChain& D, const DevA& A, uint8_t* dyn, u
         const uint8_t* st = ring + (size_t)(u % NS) * D.sp_stage_bytes;
         const int32_t* cs = (const int32_t*)st;
         const double* vs = (const double*)(st + (size_t)G * WA * 128);
-        const int64_t s = a + (int64_t)j * G;
-        const int g = (int)(b - s < (int64_t)G ? b - s : (int64_t)G);
+        const int64_t s = ((int64_t)j * NW + gw) * G;
+        const int g = (int)(ns - s < (int64_t)G ? ns - s : (int64_t)G);
         switch (WA) {
             case 3: spmv_tma_stage<3>(cs, vs, g, s, pin, wout, pw); break;
             case 4: spmv_tma_stage<4>(cs, vs, g, s, pin, wout, pw); break;

@@ -29,7 +29,7 @@ struct MArgs {
     int nrhs;                  // real right-hand sides (<= M; the rest are zero and frozen)
     const double* B;           // [nrhs][n] natural order (column-major n x nrhs)
     double* X;                 // [nrhs][n]
-    double *r, *w, *p, *z, *y, *xp;   // [npos * M] position-major
+    double *r[2], *w[2], *p[2], *z[2], *y[2], *xp[2];   // halves h of the RHS: [npos * 2] position-major
     double* partials;          // [3 M][gridDim.x]
     double* out;               // [M][4]: k, ||r_k||^2, status, -
     int nst;                   // stages per chain warp
@@ -137,8 +137,8 @@ __device__ __forceinline__ void mchunk(uint8_t* __restrict__ st, int cnt_rt, int
 // one pass (L forward or U backward) of chain c for M right-hand sides
 template <int W, bool UPPER, int KIND, int M>
 __device__ __forceinline__ void mpass(const DevChain& D, const MArgs& R, uint8_t* stages, uint64_t* full, unsigned& cq,
-                                      int c, const double* const* ops, int nv, double* out, const double (&alpha)[M],
-                                      double (&dot)[M], Scal* sc) {
+                                      int c, const double* const* ops, int nv, double* out, double* Er, double* Exp,
+                                      double* Ep, const double (&alpha)[M], double (&dot)[M], Scal* sc) {
     constexpr int RECB = 384 * W + (UPPER ? 256 : 0) + 16;
     const int lane = threadIdx.x & 31;
     const int64_t c0 = D.chain_step[c], c1 = D.chain_step[c + 1];
@@ -180,9 +180,9 @@ __device__ __forceinline__ void mpass(const DevChain& D, const MArgs& R, uint8_t
         if (!warp_ok(mbar_wait(&full[cs], cph, sc))) return;
         uint8_t* st = stages + (size_t)cs * R.stage_bytes;
         if (cnt == CC)
-            mchunk<W, UPPER, KIND, M, CC>(st, cnt, glo, out, R.r, R.xp, R.p, alpha, yprev, dot);
+            mchunk<W, UPPER, KIND, M, CC>(st, cnt, glo, out, Er, Exp, Ep, alpha, yprev, dot);
         else
-            mchunk<W, UPPER, KIND, M, 0>(st, cnt, glo, out, R.r, R.xp, R.p, alpha, yprev, dot);
+            mchunk<W, UPPER, KIND, M, 0>(st, cnt, glo, out, Er, Exp, Ep, alpha, yprev, dot);
         __syncwarp();
         if (lane == 0 && q + NST < nch) issue(q + NST, cs);
         if (++cs == (unsigned)NST) { cs = 0; cph ^= 1u; }
@@ -193,59 +193,66 @@ __device__ __forceinline__ void mpass(const DevChain& D, const MArgs& R, uint8_t
 template <bool UPPER, int KIND, int M>
 __device__ __forceinline__ void mpass_any(const DevChain& D, const MArgs& R, uint8_t* stages, uint64_t* full,
                                           unsigned& cq, int c, const double* const* ops, int nv, double* out,
-                                          const double (&alpha)[M], double (&dot)[M], Scal* sc) {
+                                          double* Er, double* Exp, double* Ep, const double (&alpha)[M],
+                                          double (&dot)[M], Scal* sc) {
     switch (UPPER ? D.W_U : D.W_L) {
-        case 1: mpass<1, UPPER, KIND, M>(D, R, stages, full, cq, c, ops, nv, out, alpha, dot, sc); break;
-        case 2: mpass<2, UPPER, KIND, M>(D, R, stages, full, cq, c, ops, nv, out, alpha, dot, sc); break;
-        default: mpass<4, UPPER, KIND, M>(D, R, stages, full, cq, c, ops, nv, out, alpha, dot, sc); break;
+        case 1: mpass<1, UPPER, KIND, M>(D, R, stages, full, cq, c, ops, nv, out, Er, Exp, Ep, alpha, dot, sc); break;
+        case 2: mpass<2, UPPER, KIND, M>(D, R, stages, full, cq, c, ops, nv, out, Er, Exp, Ep, alpha, dot, sc); break;
+        default: mpass<4, UPPER, KIND, M>(D, R, stages, full, cq, c, ops, nv, out, Er, Exp, Ep, alpha, dot, sc); break;
     }
 }
 
-// y = L^-1 r (with the fused updates of the kind) then z = U^-1 y for every chain of
-// this CTA (warp k walks chain blockIdx.x + k gridDim.x); rr / rz partial sums.
+// y = L^-1 r (with the fused updates of the kind) then z = U^-1 y.  The right-hand sides
+// come in halves of two (position-major pairs): warp k walks chain blockIdx.x + (k mod
+// per_cta) gridDim.x for half k / per_cta, so with M = 4 two warps walk each chain side
+// by side, each carrying two FMA chains per step (the records are read by both, the
+// second time from L2).  rr / rz: this thread's partial sums, zero for the other half.
 template <int KIND, int M>
 __device__ __noinline__ void mtri(const DevChain* Dp, const MArgs* Rp, uint8_t* dyn, uint64_t* bars, unsigned* cq,
                                   const double* alpha_in, double* rr, double* rz, Scal* sc) {
+    constexpr int H = M / 2;
     const DevChain& D = *Dp;
     const MArgs& R = *Rp;
     const int warp = threadIdx.x >> 5;
-    const int c = blockIdx.x + warp * gridDim.x;
-    if (warp >= D.per_cta || c >= D.nchains) return;
+    const int h = warp / D.per_cta, slot = warp % D.per_cta;
+    const int c = blockIdx.x + slot * gridDim.x;
+    if (h >= H || c >= D.nchains) return;
     uint8_t* stages = dyn + (size_t)warp * R.warp_bytes;
     uint64_t* full = bars + warp * 16;
-    double alpha[M], a[M], b[M];
+    double alpha[2], a[2], b[2];
 #pragma unroll
-    for (int m = 0; m < M; ++m) {
-        alpha[m] = alpha_in[m];
-        a[m] = rr[m];
-        b[m] = rz[m];
+    for (int j = 0; j < 2; ++j) {
+        alpha[j] = alpha_in[2 * h + j];
+        a[j] = 0.0;
+        b[j] = 0.0;
     }
     unsigned q = *cq;
     {
-        const double* ops[4] = {R.r, R.w, R.xp, R.p};
-        mpass_any<false, KIND, M>(D, R, stages, full, q, c, ops, KIND == K_ITER ? 4 : 1, R.y, alpha, a, sc);
+        const double* ops[4] = {R.r[h], R.w[h], R.xp[h], R.p[h]};
+        mpass_any<false, KIND, 2>(D, R, stages, full, q, c, ops, KIND == K_ITER ? 4 : 1, R.y[h], R.r[h], R.xp[h],
+                                  R.p[h], alpha, a, sc);
     }
     // the U pass reads y and r through TMA: order this warp's generic stores first
     asm volatile("fence.proxy.async.global;" ::: "memory");
     __syncwarp();
     {
-        const double* ops[2] = {R.y, R.r};
-        mpass_any<true, KIND, M>(D, R, stages, full, q, c, ops, 2, R.z, alpha, b, sc);
+        const double* ops[2] = {R.y[h], R.r[h]};
+        mpass_any<true, KIND, 2>(D, R, stages, full, q, c, ops, 2, R.z[h], R.r[h], R.xp[h], R.p[h], alpha, b, sc);
     }
     *cq = q;
 #pragma unroll
-    for (int m = 0; m < M; ++m) {
-        rr[m] = a[m];
-        rz[m] = b[m];
+    for (int j = 0; j < 2; ++j) {
+        rr[2 * h + j] += a[j];
+        rz[2 * h + j] += b[j];
     }
 }
 
-// w = A p for M vectors (TMA-streamed slices of uniform width WA, gathers of M values)
+// w = A p for M vectors (TMA-streamed slices of uniform width WA, gathers of the M values
+// of a neighbour from the H = M / 2 position-major halves)
 template <int WA, int M>
 __device__ __forceinline__ void mspmv_stage(const int32_t* __restrict__ cs, const double* __restrict__ vs, int g,
-                                            int64_t s, const double* __restrict__ pin, double* __restrict__ wout,
-                                            double (&pw)[M]) {
-    constexpr int G = SPCG_SPMV_G;
+                                            int64_t s, const MArgs& R, double (&pw)[M]) {
+    constexpr int G = SPCG_SPMV_G, H = M / 2;
     const int lane = threadIdx.x & 31;
 #pragma unroll
     for (int u = 0; u < G; ++u) {
@@ -258,7 +265,8 @@ __device__ __forceinline__ void mspmv_stage(const int32_t* __restrict__ cs, cons
         for (int k = 0; k < WA; ++k) {
             const int c = cs[(u * WA + k) * 32 + lane];
             vv[k] = vs[(u * WA + k) * 32 + lane];
-            ldm(pin + (int64_t)c * M, gv[k], M);
+#pragma unroll
+            for (int hh = 0; hh < H; ++hh) ldm(R.p[hh] + (int64_t)c * 2, gv[k] + 2 * hh, 2);
         }
 #pragma unroll
         for (int k = 0; k < WA; ++k)
@@ -266,31 +274,37 @@ __device__ __forceinline__ void mspmv_stage(const int32_t* __restrict__ cs, cons
             for (int m = 0; m < M; ++m) acc[m] = fma(vv[k], gv[k][m], acc[m]);
         const int64_t row = (s + u) * 32 + lane;
         double pr[M];
-        ldm(pin + row * M, pr, M);
-        stm(wout + row * M, acc, M);
+#pragma unroll
+        for (int hh = 0; hh < H; ++hh) {
+            ldm(R.p[hh] + row * 2, pr + 2 * hh, 2);
+            stm(R.w[hh] + row * 2, acc + 2 * hh, 2);
+        }
 #pragma unroll
         for (int m = 0; m < M; ++m) pw[m] = fma(pr[m], acc[m], pw[m]);
     }
 }
 
 template <int M>
-__device__ void mspmv(const DevChain& D, const DevA& A, uint8_t* dyn, uint64_t* bars, unsigned& spq,
-                      const double* __restrict__ pin, double* __restrict__ wout, double (&pw)[M], Scal* sc) {
+__device__ void mspmv(const DevChain& D, const DevA& A, uint8_t* dyn, uint64_t* bars, unsigned& spq, const MArgs& R,
+                      double (&pw)[M], Scal* sc) {
     constexpr int G = SPCG_SPMV_G;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t ns = A.nslices;
     const int64_t NW = (int64_t)gridDim.x * NWARP, gw = (int64_t)blockIdx.x * NWARP + warp;
-    const int64_t a = gw * ns / NW, b = (gw + 1) * ns / NW;
+    // groups of G slices dealt round-robin over the grid's warps (group gi = j NW + gw): the
+    // positions of weak-coupling fragments cluster at the end of the layout, and contiguous
+    // ranges left the warps that got them (far gathers) the last to reach the barrier
+    const int64_t ngr = (ns + G - 1) / G;
     const int NS = D.sp_nst, WA = D.WA;
     uint8_t* ring = dyn + (size_t)warp * NS * D.sp_stage_bytes;
     uint64_t* bar = bars + warp * 4;
-    const int nst = (int)((b - a + G - 1) / G);
+    const int nst = (int)(gw < ngr ? (ngr - gw + NW - 1) / NW : 0);
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     __syncwarp();
     auto issue = [&](int j) {
         const int slot = (spq + j) % NS;
-        const int64_t s = a + (int64_t)j * G;
-        const int g = (int)(b - s < (int64_t)G ? b - s : (int64_t)G);
+        const int64_t s = ((int64_t)j * NW + gw) * G;
+        const int g = (int)(ns - s < (int64_t)G ? ns - s : (int64_t)G);
         const unsigned cb = (unsigned)(g * WA * 128), vb = (unsigned)(g * WA * 256);
         uint8_t* st = ring + (size_t)slot * D.sp_stage_bytes;
         mbar_arrive_tx(&bar[slot], cb + vb);
@@ -305,15 +319,15 @@ __device__ void mspmv(const DevChain& D, const DevA& A, uint8_t* dyn, uint64_t* 
         const uint8_t* st = ring + (size_t)(u % NS) * D.sp_stage_bytes;
         const int32_t* cs = (const int32_t*)st;
         const double* vs = (const double*)(st + (size_t)G * WA * 128);
-        const int64_t s = a + (int64_t)j * G;
-        const int g = (int)(b - s < (int64_t)G ? b - s : (int64_t)G);
+        const int64_t s = ((int64_t)j * NW + gw) * G;
+        const int g = (int)(ns - s < (int64_t)G ? ns - s : (int64_t)G);
         switch (WA) {
-            case 3: mspmv_stage<3, M>(cs, vs, g, s, pin, wout, pw); break;
-            case 4: mspmv_stage<4, M>(cs, vs, g, s, pin, wout, pw); break;
-            case 5: mspmv_stage<5, M>(cs, vs, g, s, pin, wout, pw); break;
-            case 6: mspmv_stage<6, M>(cs, vs, g, s, pin, wout, pw); break;
-            case 7: mspmv_stage<7, M>(cs, vs, g, s, pin, wout, pw); break;
-            default: mspmv_stage<8, M>(cs, vs, g, s, pin, wout, pw); break;
+            case 3: mspmv_stage<3, M>(cs, vs, g, s, R, pw); break;
+            case 4: mspmv_stage<4, M>(cs, vs, g, s, R, pw); break;
+            case 5: mspmv_stage<5, M>(cs, vs, g, s, R, pw); break;
+            case 6: mspmv_stage<6, M>(cs, vs, g, s, R, pw); break;
+            case 7: mspmv_stage<7, M>(cs, vs, g, s, R, pw); break;
+            default: mspmv_stage<8, M>(cs, vs, g, s, R, pw); break;
         }
         __syncwarp();
         if (lane == 0 && j + NS < nst) issue(j + NS);
@@ -393,8 +407,9 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_wchain_mrhs_kernel(Params P, MA
         const int64_t pos = e / M;
         const int m = (int)(e % M);
         const int32_t row = __ldg(D.perm + pos);
-        R.r[e] = (row >= 0 && m < R.nrhs) ? R.B[(int64_t)m * n + row] : 0.0;
-        R.xp[e] = 0.0;
+        const int64_t hi = pos * 2 + (m & 1);
+        R.r[m >> 1][hi] = (row >= 0 && m < R.nrhs) ? R.B[(int64_t)m * n + row] : 0.0;
+        R.xp[m >> 1][hi] = 0.0;
     }
     sync_tma(P.sc, gen);
     double alpha[M], rr_l[M], rz_l[M];
@@ -445,7 +460,7 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_wchain_mrhs_kernel(Params P, MA
         double pw[M], zero[M];
 #pragma unroll
         for (int m = 0; m < M; ++m) { pw[m] = 0.0; zero[m] = 0.0; }
-        mspmv<M>(sD, P.A, dynw, spbar, spq, R.p, R.w, pw, P.sc);
+        mspmv<M>(sD, P.A, dynw, spbar, spq, sR, pw, P.sc);
         mpartials<M>(pw, zero, R.partials, 2 * M);
         sync_tma(P.sc, gen);
         msums<M>(R.partials, 2 * M, M, sums);
@@ -480,29 +495,24 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_wchain_mrhs_kernel(Params P, MA
                 rr[m] = sums[M + m];
             }
         }
-        {   // p = z + beta p, 16-byte accesses (M is even: a pair never straddles two rows' RHS
-            // sets), four of them in flight per thread before the first store
-            double2* __restrict__ p2 = (double2*)R.p;
-            const double2* __restrict__ z2 = (const double2*)R.z;
-            const int64_t n2 = npos * M / 2;
-            for (int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x; i < n2; i += 4 * stride) {
+        // p = z + beta p, 16-byte accesses (a position's pair of a half), four in flight per thread
+#pragma unroll
+        for (int hh = 0; hh < M / 2; ++hh) {
+            double2* __restrict__ p2 = (double2*)R.p[hh];
+            const double2* __restrict__ z2 = (const double2*)R.z[hh];
+            const double b0 = beta[2 * hh], b1 = beta[2 * hh + 1];
+            for (int64_t i = (int64_t)blockIdx.x * BLOCK + threadIdx.x; i < npos; i += 4 * stride) {
                 double2 pv[4], zv[4];
 #pragma unroll
                 for (int u = 0; u < 4; ++u)
-                    if (i + u * stride < n2) {
+                    if (i + u * stride < npos) {
                         pv[u] = p2[i + u * stride];
                         zv[u] = __ldcg(z2 + i + u * stride);
                     }
 #pragma unroll
                 for (int u = 0; u < 4; ++u)
-                    if (i + u * stride < n2) {
-                        const int64_t j = i + u * stride;
-                        double b0 = beta[0], b1 = beta[1];
-                        if constexpr (M == 4) {
-                            if ((j & 1) != 0) { b0 = beta[2]; b1 = beta[3]; }
-                        }
-                        p2[j] = make_double2(fma(b0, pv[u].x, zv[u].x), fma(b1, pv[u].y, zv[u].y));
-                    }
+                    if (i + u * stride < npos)
+                        p2[i + u * stride] = make_double2(fma(b0, pv[u].x, zv[u].x), fma(b1, pv[u].y, zv[u].y));
             }
         }
         sync_tma(P.sc, gen);
@@ -513,7 +523,7 @@ __global__ void __launch_bounds__(BLOCK, 1) spcg_wchain_mrhs_kernel(Params P, MA
         const int64_t pos = e / M;
         const int m = (int)(e % M);
         const int32_t row = __ldg(D.perm + pos);
-        if (row >= 0 && m < R.nrhs) R.X[(int64_t)m * n + row] = R.xp[e];
+        if (row >= 0 && m < R.nrhs) R.X[(int64_t)m * n + row] = R.xp[m >> 1][pos * 2 + (m & 1)];
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
 #pragma unroll
@@ -540,16 +550,19 @@ size_t spcg_mrhs_args_size() { return sizeof(MArgs); }
 // fills an MArgs at dst (kernels.cu does not see the struct)
 void spcg_mrhs_args_fill(void* dst, int nrhs, const double* B, double* X, double* const* vec, double* partials,
                          double* out, int nst, unsigned stage_bytes, unsigned warp_bytes) {
+    // vec: 12 arrays, [vector][half] for r, w, p, z, y, xp
     MArgs* a = (MArgs*)dst;
     a->nrhs = nrhs;
     a->B = B;
     a->X = X;
-    a->r = vec[0];
-    a->w = vec[1];
-    a->p = vec[2];
-    a->z = vec[3];
-    a->y = vec[4];
-    a->xp = vec[5];
+    for (int h = 0; h < 2; ++h) {
+        a->r[h] = vec[0 + h];
+        a->w[h] = vec[2 + h];
+        a->p[h] = vec[4 + h];
+        a->z[h] = vec[6 + h];
+        a->y[h] = vec[8 + h];
+        a->xp[h] = vec[10 + h];
+    }
     a->partials = partials;
     a->out = out;
     a->nst = nst;

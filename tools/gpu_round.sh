@@ -23,6 +23,7 @@ if has bench; then
     timeout 600 python bench.py --workload $W --steps 5 --warmup 3 --no-cpu-baseline > "$O/bench_${W,,}.json" 2> "$O/bench_${W,,}.err"
   done
   timeout 900 python bench.py --workload C5 --steps 3 --warmup 3 > "$O/bench_c5.json" 2> "$O/bench_c5.err"
+  timeout 900 python bench.py --impl reference --steps 2 --warmup 3 > "$O/bench_ref_c4.json" 2> "$O/bench_ref_c4.err"
 fi
 if has ncu; then
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file "$O/launches_c4.csv" \
@@ -30,5 +31,13 @@ if has ncu; then
   # one forced-k (20 iterations) C4 solve: skip the converged solve that exp_iter runs first
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:spcg_ -s 1 -c 1 -f -o "$O/prof_c4" \
     python tools/exp_iter.py aniso_layered 4096 4096 4 --k 20 --modes alg2 --reps 1 > "$O/ncu_full.log" 2>&1
+  # the report itself is ~50 MB (over gpurun's copy-back limit): export the pages, keep the report off gpurun_out
+  if [ -f "$O/prof_c4.ncu-rep" ]; then
+    ncu -i "$O/prof_c4.ncu-rep" --page raw --csv > "$O/prof_c4_raw.csv" 2>/dev/null
+    ncu -i "$O/prof_c4.ncu-rep" --page details --csv > "$O/prof_c4_details.csv" 2>/dev/null
+    ncu -i "$O/prof_c4.ncu-rep" --page source --csv --print-source sass > "$O/prof_c4_sass.csv" 2>/dev/null
+    gzip -f "$O/prof_c4_sass.csv"
+    mv "$O/prof_c4.ncu-rep" /tmp/prof_c4.ncu-rep
+  fi
 fi
 echo done > "$O/DONE"

@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Summarise an ncu report (--set full) and a launch list into profiles/.
 
-usage: tools/ncu_summary.py REPORT.ncu-rep LAUNCHES.csv OUT.md --workload C2 --impl spcg [--json profiles/ncu_summary.json]
+usage: tools/ncu_summary.py REPORT.ncu-rep|RAW.csv LAUNCHES.csv OUT.md --workload C2 --impl spcg [--json profiles/ncu_summary.json]
 """
 import argparse, csv, io, json, os, subprocess, sys
 
@@ -13,7 +13,12 @@ UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
 
 
 def raw(rep):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    """REPORT.ncu-rep, or the CSV of its raw page (`ncu -i REP --page raw --csv`)."""
+    if rep.endswith(".csv"):
+        out = open(rep).read()
+    else:
+        out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    out = "".join(l + "\n" for l in out.splitlines() if not l.startswith("=="))
     rows = list(csv.reader(io.StringIO(out)))
     return rows[0], rows[1], rows[2:]
 
