@@ -264,7 +264,7 @@ def main():
 
     # NEXT-1: ILU(0) systems are set up on the GPU (validation, Algorithm 2, ILU(0), level
     # sets: gsetup.cu); the host setup of the same products is timed once for comparison
-    setup_kind = "gpu" if K == 0 else "host"
+    setup_kind = "gpu" if K == 0 and A.n >= 65536 else "host"     # tiny systems: the host is quicker
     handles = {}
     for mode in ("alg2", "none"):
         handles[mode] = spcg.SPCG(A, mode=mode, K=K, sptrsv=args.sptrsv, parts=args.parts, device=dev, stream=stream,

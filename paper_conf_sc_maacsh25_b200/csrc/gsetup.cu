@@ -573,13 +573,15 @@ spcg_status_t levels(Ctx& C, const GCsr& M, const uint8_t* drop, bool lower, int
 // Host <-> device copies of pageable std::vector data through two pinned bounce
 // buffers (a pageable cudaMemcpy runs at a few GB/s; this overlaps the host memcpy of
 // one chunk with the DMA of the other).
-constexpr size_t BOUNCE = 32u << 20;
+constexpr size_t BOUNCE_MAX = 32u << 20;
 struct Bounce {
     void* buf[2] = {nullptr, nullptr};
     cudaEvent_t ev[2] = {nullptr, nullptr};
     bool ok = false;
-    Bounce() {
-        ok = cudaMallocHost(&buf[0], BOUNCE) == cudaSuccess && cudaMallocHost(&buf[1], BOUNCE) == cudaSuccess &&
+    size_t size = 0;            // bytes per buffer: the largest copy, at most BOUNCE_MAX
+    explicit Bounce(size_t largest) {
+        size = std::max<size_t>(4096, std::min(BOUNCE_MAX, largest));
+        ok = cudaMallocHost(&buf[0], size) == cudaSuccess && cudaMallocHost(&buf[1], size) == cudaSuccess &&
              cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming) == cudaSuccess &&
              cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming) == cudaSuccess;
     }
@@ -597,7 +599,7 @@ spcg_status_t h2d(Ctx& C, Bounce& B, void* dst, const void* src, size_t bytes) {
     }
     size_t off = 0;
     for (int k = 0; off < bytes; k ^= 1) {
-        const size_t m = std::min(BOUNCE, bytes - off);
+        const size_t m = std::min(B.size, bytes - off);
         GCK(cudaEventSynchronize(B.ev[k]));                  // the DMA out of this buffer is done
         std::memcpy(B.buf[k], (const char*)src + off, m);
         GCK(cudaMemcpyAsync((char*)dst + off, B.buf[k], m, cudaMemcpyHostToDevice, C.s));
@@ -613,15 +615,15 @@ spcg_status_t d2h(Ctx& C, Bounce& B, void* dst, const void* src, size_t bytes) {
         return SPCG_OK;
     }
     // chunk j lands in buffer j & 1; it is drained while chunk j + 1 is in flight
-    const size_t nch = (bytes + BOUNCE - 1) / BOUNCE;
+    const size_t nch = (bytes + B.size - 1) / B.size;
     for (size_t j = 0; j < nch + 1; ++j) {
         if (j < nch) {
-            const size_t off = j * BOUNCE, m = std::min(BOUNCE, bytes - off);
+            const size_t off = j * B.size, m = std::min(B.size, bytes - off);
             GCK(cudaMemcpyAsync(B.buf[j & 1], (const char*)src + off, m, cudaMemcpyDeviceToHost, C.s));
             GCK(cudaEventRecord(B.ev[j & 1], C.s));
         }
         if (j > 0) {
-            const size_t i = j - 1, off = i * BOUNCE, m = std::min(BOUNCE, bytes - off);
+            const size_t i = j - 1, off = i * B.size, m = std::min(B.size, bytes - off);
             GCK(cudaEventSynchronize(B.ev[i & 1]));
             std::memcpy((char*)dst + off, B.buf[i & 1], m);
         }
@@ -765,7 +767,7 @@ spcg_status_t gpu_setup_k0(const Csr& Ain, const spcg_drop_params_t& p, int devi
         set_error("gpu setup: device allocation failed");
         return SPCG_ERR_OOM;
     }
-    Bounce B;
+    Bounce B((size_t)8 * std::max<int64_t>(nnz, n + 1));
     spcg_status_t st;
     if ((st = h2d(C, B, A.rp, Ain.rp.data(), 8 * (n + 1))) != SPCG_OK) return st;
     if ((st = h2d(C, B, A.col, Ain.col.data(), 4 * nnz)) != SPCG_OK) return st;
