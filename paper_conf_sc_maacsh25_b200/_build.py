@@ -41,7 +41,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     jobs = []
     for cu in sorted(glob.glob(os.path.join(CSRC, "*.cu"))):
         o = os.path.join(bdir, os.path.basename(cu) + ".o")
-        cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
+        cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fopenmp", "-Xptxas", "-v",
                "-I", os.path.join(ROOT, "include"), *defines, "-c", cu, "-o", o]
         jobs.append((cu, o, cmd))
     for cpp in sorted(glob.glob(os.path.join(CSRC, "*.cpp"))):

@@ -32,11 +32,6 @@ __device__ __forceinline__ void cpa16(void* sdst, const void* gsrc) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(sdst)), "l"(gsrc) : "memory");
 }
 __device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-// the mbarrier's pending count is raised by one now and lowered when this thread's
-// earlier cp.async copies have landed
-__device__ __forceinline__ void cpa_mbar_arrive(uint64_t* b) {
-    asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" ::"r"(smem_u32(b)) : "memory");
-}
 __device__ __forceinline__ void cpa_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 __device__ __forceinline__ void cpa_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 // generic-proxy global writes -> later TMA (async-proxy) reads of the same data
@@ -341,35 +336,17 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
     auto next_slot = [&](unsigned& slot, unsigned& ph) {
         if (++slot == (unsigned)NST) { slot = 0; ph ^= 1u; }
     };
-    // Stage fill.  Shuffle-only passes (!GEN): the whole warp copies the chunk with 16-byte
-    // cp.async (each lane every 32nd piece) and arrives on the stage mbarrier through
-    // cp.async.mbarrier.arrive — no single-lane section: issuing ~5 bulk copies from one
-    // lane cost as much as the chunk's 8 steps (R2UR + elect per copy, ncu source view,
-    // DESIGN.md §5.5).  GEN passes keep TMA bulk copies from lane 0 (their flag prefetch
-    // counts cp.async groups).  Called by all lanes in both cases.
-    auto issue = [&](int q, unsigned slot) {
+    auto issue = [&](int q, unsigned slot) {               // lane 0 only
         int64_t glo;
         int cnt;
         chunk_range(q, glo, cnt);
         uint8_t* st = stage_at(slot);
         const unsigned rb = (unsigned)(cnt * RECB), vb = (unsigned)cnt * 256u;
+        mbar_arrive_tx(&WS.full[slot], rb + vb * ops.nv);
+        bulk_g2s(st, recs + (size_t)glo * RECB, rb, &WS.full[slot]);
         uint8_t* vdst = st + (size_t)CC * RECB;
-        if constexpr (!GEN) {
-            const uint8_t* rs = recs + (size_t)glo * RECB;
-            for (unsigned off = 16u * lane; off < rb; off += 512u) cpa16(st + off, rs + off);
-            for (int v = 0; v < ops.nv; ++v) {
-                const uint8_t* vs = (const uint8_t*)(ops.v[v] + 32 * glo);
-                for (unsigned off = 16u * lane; off < vb; off += 512u) cpa16(vdst + (size_t)v * CC * 256 + off, vs + off);
-            }
-            cpa_mbar_arrive(&WS.full[slot]);
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&WS.full[slot]);
-        } else if (lane == 0) {
-            mbar_arrive_tx(&WS.full[slot], rb + vb * ops.nv);
-            bulk_g2s(st, recs + (size_t)glo * RECB, rb, &WS.full[slot]);
-            for (int v = 0; v < ops.nv; ++v)
-                bulk_g2s(vdst + (size_t)v * CC * 256, ops.v[v] + 32 * glo, vb, &WS.full[slot]);
-        }
+        for (int v = 0; v < ops.nv; ++v)
+            bulk_g2s(vdst + (size_t)v * CC * 256, ops.v[v] + 32 * glo, vb, &WS.full[slot]);
     };
     auto wait_at = [&](uint64_t* bars, unsigned slot, unsigned ph) -> bool {
         return warp_ok(mbar_wait(&bars[slot], ph, E.sc));
@@ -438,7 +415,7 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
     GenCtx G{WS.hist, WS.extq, mb, E.sc, ep, GEN && (cfl & (UPPER ? CC_UHIST : CC_LHIST)) != 0};
     const bool rsrc_is_r = ops.v[0] == E.r;
     const unsigned sl0 = cq % (unsigned)NST, ph0 = (cq / (unsigned)NST) & 1u;
-    if (ROLE != 2) {
+    if (ROLE != 2 && lane == 0) {
         unsigned sl = sl0, ph = ph0;
         for (int q = 0; q < min(NST, nch); ++q) {
             issue(q, sl);
@@ -465,10 +442,9 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
             if (!wait_at(UPPER ? WS.hand : WS.full, cs, cph)) return;
             help_chunk<UPPER, KIND>(st, RECB, cnt, glo, ops.nv, rsrc_is_r, E.use_x0, out, E.r, E.xp, E.p, alpha, dot);
             __syncwarp();
-            if (!UPPER) {
-                if (lane == 0) mbar_arrive(&WS.hand[cs]);
-            } else if (q + NST < nch) {
-                issue(q + NST, cs);
+            if (lane == 0) {
+                if (!UPPER) mbar_arrive(&WS.hand[cs]);
+                else if (q + NST < nch) issue(q + NST, cs);
             }
             cs = ns_;
             cph = nph;
@@ -498,8 +474,10 @@ __device__ __forceinline__ void chain_pass(const DevChain& D, const PassEnv& E, 
             run_chunk<W, UPPER, KIND, GEN, SPLIT, 0, VB>(st, cnt, glo, q * CC, ops.nv, rsrc_is_r, E.use_x0, out, E.r,
                                                          E.xp, E.p, alpha, yprev, dot, G);
         __syncwarp();
-        if (SPLIT && UPPER && lane == 0) mbar_arrive(&WS.hand[cs]);
-        if (refill && q + NST < nch) issue(q + NST, cs);
+        if (lane == 0) {
+            if (SPLIT && UPPER) mbar_arrive(&WS.hand[cs]);
+            if (refill && q + NST < nch) issue(q + NST, cs);
+        }
         cs = ns_;
         cph = nph;
     }
