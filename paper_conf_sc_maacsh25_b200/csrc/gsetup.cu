@@ -75,8 +75,9 @@ __global__ void k_validate(int64_t n, const int64_t* __restrict__ rp, const int3
     unsigned long long nl = 0, c = 0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const int64_t q0 = rp[i], q1 = rp[i + 1];
+        const int64_t nnz = rp[n];
         unsigned code = 0;
-        if (q1 < q0) code = E_ROWPTR;
+        if (q1 < q0 || q0 < 0 || q1 > nnz) code = E_ROWPTR;      // never read outside col / val
         bool diag = false;
         int64_t prev = -1;
         for (int64_t q = q0; q < q1 && !code; ++q) {
@@ -98,7 +99,7 @@ __global__ void k_validate(int64_t n, const int64_t* __restrict__ rp, const int3
             for (int64_t q = q0; q < q1; ++q) {
                 const int64_t j = col[q];
                 int64_t lo = rp[j], hi = rp[j + 1] - 1;
-                if (hi < lo || rp[j + 1] < rp[j]) { code = E_PATTERN; break; }
+                if (hi < lo || lo < 0 || rp[j + 1] > nnz) { code = E_PATTERN; break; }
                 int64_t found = -1;
                 while (lo <= hi) {
                     const int64_t mid = (lo + hi) >> 1;

@@ -44,7 +44,7 @@ spcg_status_t validate_and_mirror(const Csr& A, std::vector<int64_t>& pos_t) {
     if (nnz >= (int64_t(1) << 31)) { set_error("nnz >= 2^31"); return SPCG_ERR_BAD_MATRIX; }
     std::vector<int64_t> cnt(n + 1, 0);
     for (int64_t i = 0; i < n; ++i) {
-        if (A.rp[i + 1] < A.rp[i]) { set_error("row_ptr not monotone"); return SPCG_ERR_BAD_MATRIX; }
+        if (A.rp[i + 1] < A.rp[i] || A.rp[i + 1] > nnz) { set_error("row_ptr not monotone"); return SPCG_ERR_BAD_MATRIX; }
         bool diag = false;
         int64_t prev = -1;
         for (int64_t q = A.rp[i]; q < A.rp[i + 1]; ++q) {

@@ -111,6 +111,13 @@ def test_gpu_setup_errors():
     with pytest.raises(lib.SpcgError) as e:
         lib.SPCG(gen.CSR(A.n, A.row_ptr, A.col, val), setup="gpu")
     assert e.value.status == lib.ERR_BAD_MATRIX
+    # a row pointer that runs past nnz then back (rp[n] == nnz still): no out-of-range read
+    rp = A.row_ptr.copy()
+    rp[3] = rp[-1] + 5
+    for setup in ("gpu", "host"):
+        with pytest.raises(lib.SpcgError) as e:
+            lib.SPCG(gen.CSR(A.n, rp, A.col, A.val), setup=setup)
+        assert e.value.status == lib.ERR_BAD_MATRIX
     # zero pivot: [[1, 1], [1, 1]] has u_11 = 1 - 1 = 0; the host reports the same row
     Z = gen.CSR(2, np.array([0, 2, 4], np.int64), np.array([0, 1, 0, 1], np.int32), np.ones(4))
     for setup in ("gpu", "host"):
