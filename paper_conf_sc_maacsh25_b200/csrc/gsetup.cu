@@ -910,7 +910,9 @@ spcg_status_t gpu_setup_k0(const Csr& Ain, const spcg_drop_params_t& p, int devi
     // levels of the factors (O8); L's give the row order of the numeric factorisation
     F.levL.resize(n);
     F.levU.resize(n);
-    if ((st = levels(C, Ld, nullptr, true, lev, &F.wL)) != SPCG_OK) return st;
+    // K = 0: the pattern of L_s is the strictly-lower part of Ahat, so L's levels are the
+    // ones Algorithm 2 just computed for the chosen Ahat (still in lev): no second pass
+    F.wL = sp.w_Ahat;
     {
         int32_t* order = C.pool.get<int32_t>(n);
         int* done = C.pool.get<int>(n);

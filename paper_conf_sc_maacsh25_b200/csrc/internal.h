@@ -33,8 +33,8 @@ using fast_vector = std::vector<T, NoInit<T>>;
 struct Csr {                       // host CSR, int64 row pointers
     int64_t n = 0;
     std::vector<int64_t> rp;
-    std::vector<int32_t> col;
-    std::vector<double> val;
+    fast_vector<int32_t> col;      // resize() leaves entries uninitialised: every builder writes them all
+    fast_vector<double> val;
     int64_t nnz() const { return rp.empty() ? 0 : rp.back(); }
 };
 

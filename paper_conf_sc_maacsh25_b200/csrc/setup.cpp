@@ -340,8 +340,8 @@ spcg_status_t iluk_symbolic(const Csr& Ah, int K, Factors& F) {
                 lcol[dst] = (int32_t)i; llev[dst] = ulev[q];
             }
     }
-    F.L.n = n; F.L.rp = std::move(lrp); F.L.col = std::move(lcol); F.L.val.assign(F.L.col.size(), 0.0);
-    F.U.n = n; F.U.rp = std::move(urp); F.U.col = std::move(ucol); F.U.val.assign(F.U.col.size(), 0.0);
+    F.L.n = n; F.L.rp = std::move(lrp); F.L.col.assign(lcol.begin(), lcol.end()); F.L.val.assign(F.L.col.size(), 0.0);
+    F.U.n = n; F.U.rp = std::move(urp); F.U.col.assign(ucol.begin(), ucol.end()); F.U.val.assign(F.U.col.size(), 0.0);
     F.fill_level.resize(F.L.col.size() + F.U.col.size());
     int64_t o = 0;
     for (int64_t i = 0; i < n; ++i) {
