@@ -678,30 +678,19 @@ __device__ void chain_spmv_tma(const DevChain& D, const DevA& A, uint8_t* dyn, u
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t ns = A.nslices;
     const int64_t NW = (int64_t)gridDim.x * NWARP, gw = (int64_t)blockIdx.x * NWARP + warp;
-    // blocks of SPMV_BG groups of G slices dealt round-robin over the grid's warps: the
+    // groups of G slices dealt round-robin over the grid's warps (group gi = j NW + gw): the
     // positions of weak-coupling fragments cluster at the end of the layout, and contiguous
-    // ranges left the warps that got them (far gathers) the last to reach the barrier;
-    // a block keeps neighbouring slices on one warp (the p gathers of a slice's stencil
-    // neighbours, one step before / after, then hit L1)
-    constexpr int BG = 8;
+    // ranges left the warps that got them (far gathers) the last to reach the barrier
     const int64_t ngr = (ns + G - 1) / G;
-    const int64_t nbl = (ngr + BG - 1) / BG;
-    auto group_of = [&](int j) -> int64_t { return ((int64_t)(j / BG) * NW + gw) * BG + (j % BG); };
     const int NS = D.sp_nst, WA = D.WA;
     uint8_t* ring = dyn + (size_t)warp * NS * D.sp_stage_bytes;
     uint64_t* bar = bars + warp * 4;
-    // stages of this warp: full blocks, then the part of its last block inside the range
-    int nst = 0;
-    if (gw < nbl) {
-        const int64_t myb = (nbl - gw + NW - 1) / NW;               // blocks of this warp
-        const int64_t lastg = ((myb - 1) * NW + gw) * BG;           // first group of its last block
-        nst = (int)((myb - 1) * BG + (ngr - lastg < BG ? ngr - lastg : (int64_t)BG));
-    }
+    const int nst = (int)(gw < ngr ? (ngr - gw + NW - 1) / NW : 0);
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic reads of this smem done
     __syncwarp();
     auto issue = [&](int j) {
         const int slot = (spq + j) % NS;
-        const int64_t s = group_of(j) * G;
+        const int64_t s = ((int64_t)j * NW + gw) * G;
         const int g = (int)(ns - s < (int64_t)G ? ns - s : (int64_t)G);
         const unsigned cb = (unsigned)(g * WA * 128), vb = (unsigned)(g * WA * 256);
         uint8_t* st = ring + (size_t)slot * D.sp_stage_bytes;
@@ -720,7 +709,7 @@ __device__ void chain_spmv_tma(const DevChain& D, const DevA& A, uint8_t* dyn, u
         const uint8_t* st = ring + (size_t)(u % NS) * D.sp_stage_bytes;
         const int32_t* cs = (const int32_t*)st;
         const double* vs = (const double*)(st + (size_t)G * WA * 128);
-        const int64_t s = group_of(j) * G;
+        const int64_t s = ((int64_t)j * NW + gw) * G;
         const int g = (int)(ns - s < (int64_t)G ? ns - s : (int64_t)G);
         switch (WA) {
             case 3: spmv_tma_stage<3>(cs, vs, g, s, pin, wout, pw); break;
