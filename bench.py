@@ -635,6 +635,9 @@ def run_batch(args, ws, rank, local):
                 "lpt_projection_note": "LPT over the measured per-system solve times (concurrent lanes: each "
                                        "system's own event time); the largest system bounds the 8-GPU makespan",
                 "largest_system_ms": max(meas.values()),
+                # the largest system alone bounds the 8-GPU makespan, so strong scaling
+                # cannot beat T_N / (8 max_i T_i) with T_N this run's makespan at N GPUs
+                "efficiency_bound_8gpu": (ms * ws) / (8.0 * max(meas.values())),
                 "per_system": [[r.index, r.family, r.n, r.iterations, round(r.iter_phase_ms, 3), r.chosen_pct,
                                 r.status] for r in allr],
                 "lpt_load_balance": max(load) / (sum(load) / ws)}

@@ -74,7 +74,8 @@ enum {
     SPCG_DROP_FIXED = 1,            /* Ahat = A - S_t with t = fixed_pct */
     SPCG_DROP_WAVEFRONT_AWARE = 2   /* Algorithm 2 over ratios_pct (default {10,5,1}) */
 };
-enum { SPCG_NORM_FRO = 0, SPCG_NORM_INF = 1 };          /* reading A6 of ||Ahat||_2, ||S|| */
+enum { SPCG_NORM_FRO = 0, SPCG_NORM_INF = 1,            /* reading A6 of ||Ahat||_2, ||S|| */
+       SPCG_NORM_SPECTRAL = 2 };                        /* power method, 100 steps from (1..1) (host setup) */
 enum { SPCG_DENOM_WA = 0, SPCG_DENOM_WAHAT = 1 };       /* reading A8: Eq. 7 vs Alg. 2 line 10 */
 
 typedef struct {

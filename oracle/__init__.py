@@ -64,6 +64,8 @@ def _load():
         lib.or_norm_fro.restype = ctypes.c_double
         lib.or_norm_inf.argtypes = [CP]
         lib.or_norm_inf.restype = ctypes.c_double
+        lib.or_norm_spec.argtypes = [CP]
+        lib.or_norm_spec.restype = ctypes.c_double
         lib.or_alg2.argtypes = [CP, P, ctypes.c_int, ctypes.c_double, ctypes.c_double, ctypes.c_int,
                                 ctypes.c_int, CP, P, P, P]
         lib.or_iluk_symbolic.argtypes = [CP, ctypes.c_int, CP, ctypes.POINTER(ctypes.POINTER(ctypes.c_int32))]
@@ -146,6 +148,11 @@ def indicator(Ahat: CSR, S: CSR, norm_reading: int = 0):
     out = np.zeros(3)
     v = _load().or_indicator(ctypes.byref(_in(Ahat)), ctypes.byref(_in(S)), norm_reading, _p(out))
     return float(v), dict(kappa=out[0], inv_norm=out[1], s_norm=out[2])
+
+
+def norm_spec(M: CSR) -> float:
+    """SPECTRAL reading of ||M||_2: the power method, 100 steps from the all-ones vector."""
+    return float(_load().or_norm_spec(ctypes.byref(_in(M))))
 
 
 def alg2(A: CSR, ratios=(10.0, 5.0, 1.0), tau=1.0, omega=10.0, norm_reading=0, denom_mode=0):

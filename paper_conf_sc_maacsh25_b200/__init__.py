@@ -204,7 +204,7 @@ def drop_params(mode="alg2", fixed_pct=0.0, ratios=(10.0, 5.0, 1.0), tau=1.0, om
         p.ratios_pct[i] = r
     p.tau = tau
     p.omega_pct = omega
-    p.norm_reading = {"fro": 0, "inf": 1}[norm]
+    p.norm_reading = {"fro": 0, "inf": 1, "spectral": 2}[norm]
     p.reduction_denominator = {"w_A": 0, "w_Ahat": 1}[denominator]
     return p
 

@@ -113,6 +113,10 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
     spcg_drop_params_t drop;
     if (drop_in) drop = *drop_in; else spcg_drop_params_default(&drop);
     if (drop.mode < 0 || drop.mode > 2) { set_error("bad drop mode"); return SPCG_ERR_INVALID_ARG; }
+    if (drop.norm_reading < 0 || drop.norm_reading > SPCG_NORM_SPECTRAL) {
+        set_error("bad norm_reading");
+        return SPCG_ERR_INVALID_ARG;
+    }
     spcg_options_t opt;
     if (opt_in) opt = *opt_in; else spcg_options_default(&opt);
     if (opt.exec == SPCG_EXEC_GRAPH_WHILE) {
@@ -146,7 +150,9 @@ spcg_status_t spcg_setup(const spcg_csr_t* Ain, const spcg_drop_params_t* drop_i
             set_error("bad setup_device");
             return SPCG_ERR_INVALID_ARG;
         }
-        const bool on_gpu = opt.setup_device == SPCG_SETUP_GPU && K == 0 && opt.device >= 0;
+        // the GPU setup covers ILU(0) with the FRO / INF readings; SPECTRAL runs on the host
+        const bool on_gpu = opt.setup_device == SPCG_SETUP_GPU && K == 0 && opt.device >= 0 &&
+                            (drop.mode != SPCG_DROP_WAVEFRONT_AWARE || drop.norm_reading != SPCG_NORM_SPECTRAL);
         double t1, t2, t3, t4;
         spcg_status_t st;
         if (on_gpu) {

@@ -169,6 +169,31 @@ static Csr apply_drop(const Csr& A, const std::vector<int64_t>& pos_t, const std
 // Indicator of Alg. 2 lines 4-5: kappa ~ ||Ahat||_inf / min diag, ||Ahat^-1|| ~
 // kappa / ||Ahat||_2, value ||Ahat^-1|| * ||S||; norms per reading A6, summed in
 // row-major order.
+// SPECTRAL reading (A6, SPCG_NORM_SPECTRAL): ||M||_2 by the power method — v_0 =
+// (1..1)/sqrt(n), w = M v_k in CSR order, v_{k+1} = w / ||w||_2, 100 steps, the last
+// ||w||_2 — with M = Ahat (keep = 1: entries not dropped) or S (keep = 0: the dropped
+// ones) read straight from A and the mask (the same order as their compacted CSR).
+static double norm_spec(const Csr& A, const std::vector<uint8_t>& drop, int keep) {
+    const int64_t n = A.n;
+    std::vector<double> v(n, 1.0 / std::sqrt((double)n)), w(n);
+    double est = 0.0;
+    for (int k = 0; k < 100; ++k) {
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < n; ++i) {
+            double acc = 0.0;
+            for (int64_t q = A.rp[i]; q < A.rp[i + 1]; ++q)
+                if ((drop[q] == 0) == (keep == 1)) acc += A.val[q] * v[A.col[q]];
+            w[i] = acc;
+        }
+        double ss = 0.0;
+        for (int64_t i = 0; i < n; ++i) ss += w[i] * w[i];
+        est = std::sqrt(ss);
+        if (est == 0.0) break;
+        for (int64_t i = 0; i < n; ++i) v[i] = w[i] / est;
+    }
+    return est;
+}
+
 static double indicator(const Csr& A, const std::vector<uint8_t>& drop, int norm_reading) {
     double fro_h = 0.0, fro_s = 0.0, inf_h = 0.0, inf_s = 0.0, mind = INFINITY;
     for (int64_t i = 0; i < A.n; ++i) {
@@ -185,8 +210,10 @@ static double indicator(const Csr& A, const std::vector<uint8_t>& drop, int norm
         if (rs > inf_s) inf_s = rs;
     }
     double kappa = inf_h / mind;
-    double a2 = norm_reading == SPCG_NORM_INF ? inf_h : std::sqrt(fro_h);
-    double s = norm_reading == SPCG_NORM_INF ? inf_s : std::sqrt(fro_s);
+    double a2 = norm_reading == SPCG_NORM_INF ? inf_h
+                : norm_reading == SPCG_NORM_SPECTRAL ? norm_spec(A, drop, 1) : std::sqrt(fro_h);
+    double s = norm_reading == SPCG_NORM_INF ? inf_s
+               : norm_reading == SPCG_NORM_SPECTRAL ? norm_spec(A, drop, 0) : std::sqrt(fro_s);
     double inv = kappa / a2;
     return inv * s;
 }

@@ -314,3 +314,25 @@ def test_pcg_breakdown_branch_pin():
     assert U.val[U.row_ptr[1]] == -3.0                      # negative pivot: allowed (A12)
     r = oracle.pcg(A, L, U, b, 1e-10, 10)
     assert r["status"] == oracle.BREAKDOWN and r["k"] == 0 and not np.any(r["x"])
+
+
+def test_norm_spec_power_method_pins():
+    """SPECTRAL reading of ||M||_2 (A6 option; Alg. 2 line 4 writes the 2-norm):
+    the oracle's 100-step power method against numpy's exact 2-norm.  With a spectral
+    gap it converges to it; without one it stays a lower bound (||M v|| <= ||M|| ||v||)."""
+    import numpy as np
+    # diagonal with a gap, one dominant NEGATIVE eigenvalue (symmetric indefinite, like S)
+    for d in (np.array([1.0, 2.0, 3.0, 9.0, 100.0]), np.array([-50.0, 1.0, 2.0, 3.0])):
+        M = gen.from_dense(np.diag(d))
+        assert abs(oracle.norm_spec(M) - np.abs(d).max()) <= 1e-12 * np.abs(d).max()
+    # SPD with a dominant direction: I + 10 u u^T (exact norm 1 + 10 |u|^2)
+    rng = np.random.default_rng(3)
+    u = rng.standard_normal(8)
+    D = np.eye(8) + 10.0 * np.outer(u, u)
+    ex = np.linalg.norm(D, 2)
+    assert abs(oracle.norm_spec(gen.from_dense(D)) - ex) <= 1e-10 * ex
+    # Poisson (small gap): a lower bound, already close
+    A = gen.make("poisson2d", 12, 12)
+    ex = np.linalg.norm(A.to_scipy().toarray(), 2)
+    est = oracle.norm_spec(A)
+    assert est <= ex * (1 + 1e-14) and est >= 0.9 * ex

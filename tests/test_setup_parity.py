@@ -182,3 +182,19 @@ def test_resident_executor_host_checks():
     h.close()
     with pytest.raises(lib.SpcgError):
         lib.SPCG(gen.make("poisson2d", 65, 64), sptrsv="resident", device=-1)
+
+
+@pytest.mark.parametrize("fam,params", [("aniso_layered", (96, 80, 4)), ("poisson2d", (20, 20))])
+def test_setup_spectral_reading_bit_exact(fam, params):
+    """The SPECTRAL reading of the indicator norms (power method, 100 steps) gives the
+    oracle's Algorithm 2 trace bit for bit (same operations, same order)."""
+    A = gen.make(fam, *params)
+    h = lib.SPCG(A, mode="alg2", K=0, device=-1, norm="spectral")
+    Ah, idx, tr, wA = oracle.alg2(A, norm_reading=2)
+    assert h.info["chosen_pct"] == [10.0, 5.0, 1.0][idx]
+    assert h.info["n_tried"] == len(tr)
+    for k, x in enumerate(tr):
+        assert h.info["indicator"][k] == x["ind"]
+        assert h.info["tried_w"][k] == x["w"]
+    assert np.array_equal(h.export("ahat_col"), Ah.col)
+    h.close()
