@@ -637,7 +637,16 @@ spcg_status_t h2d(Ctx& C, Bounce& B, void* dst, const void* src, size_t bytes) {
     for (int k = 0; off < bytes; k ^= 1) {
         const size_t m = std::min(B.size, bytes - off);
         GCK(cudaEventSynchronize(B.ev[k]));                  // the DMA out of this buffer is done
-        std::memcpy(B.buf[k], (const char*)src + off, m);
+        {
+            char* bd = (char*)B.buf[k];
+            const char* sp = (const char*)src + off;
+            const int64_t nb = (int64_t)((m + (1u << 20) - 1) >> 20);
+#pragma omp parallel for schedule(static)
+            for (int64_t b = 0; b < nb; ++b) {
+                const size_t o = (size_t)b << 20;
+                std::memcpy(bd + o, sp + o, std::min<size_t>(1u << 20, m - o));
+            }
+        }
         GCK(cudaMemcpyAsync((char*)dst + off, B.buf[k], m, cudaMemcpyHostToDevice, C.s));
         GCK(cudaEventRecord(B.ev[k], C.s));
         off += m;

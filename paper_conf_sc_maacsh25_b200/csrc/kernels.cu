@@ -1479,6 +1479,10 @@ struct spcg_device_s {
     double* hist = nullptr;        // residual history buffer (grown on demand, reused)
     double* stage = nullptr;       // [2n] device copies of host b, x (SPCG_HOST_PTRS), allocated once
     long long hist_cap = 0;
+    // setup-time upload: two pinned bounce buffers (the layouts are GBs of pageable
+    // std::vector data; a pageable cudaMemcpy runs at a few GB/s), released after create
+    void* ub[2] = {nullptr, nullptr};
+    cudaEvent_t uev[2] = {nullptr, nullptr};
     // multi-RHS (NEXT-4, wchain_mrhs.cu): six position-major vectors of npos x mr_M, grown on demand
     int mr_M = 0;
     double* mr_vec[12] = {};       // [vector r, w, p, z, y, xp][half]
@@ -1527,12 +1531,58 @@ static void dev_free(spcg_device_t* d, void* p) {
         }
 }
 
+constexpr size_t UP_BOUNCE = 32u << 20;
+// large arrays through the pinned bounce buffers (chunk k: parallel memcpy into buffer
+// k & 1 once its previous DMA is done, then an async copy on the handle's stream)
+static spcg_status_t h2d_bounced(spcg_device_t* d, void* dst, const void* src, size_t bytes) {
+    if (!d->ub[0]) {
+        if (cudaMallocHost(&d->ub[0], UP_BOUNCE) != cudaSuccess || cudaMallocHost(&d->ub[1], UP_BOUNCE) != cudaSuccess ||
+            cudaEventCreateWithFlags(&d->uev[0], cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&d->uev[1], cudaEventDisableTiming) != cudaSuccess) {
+            CK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, d->stream));   // no pinned memory: direct
+            return SPCG_OK;
+        }
+    }
+    size_t off = 0;
+    for (int k = 0; off < bytes; k ^= 1) {
+        const size_t m = std::min(UP_BOUNCE, bytes - off);
+        CK(cudaEventSynchronize(d->uev[k]));
+        char* bd = (char*)d->ub[k];
+        const char* sp = (const char*)src + off;
+        const int64_t nb = (int64_t)((m + (1u << 20) - 1) >> 20);
+#pragma omp parallel for schedule(static)
+        for (int64_t b = 0; b < nb; ++b) {
+            const size_t o = (size_t)b << 20;
+            std::memcpy(bd + o, sp + o, std::min<size_t>(1u << 20, m - o));
+        }
+        CK(cudaMemcpyAsync((char*)dst + off, bd, m, cudaMemcpyHostToDevice, d->stream));
+        CK(cudaEventRecord(d->uev[k], d->stream));
+        off += m;
+    }
+    return SPCG_OK;
+}
+static void release_bounce(spcg_device_t* d) {
+    if (d->ub[0] || d->ub[1]) cudaStreamSynchronize(d->stream);
+    for (int k = 0; k < 2; ++k) {
+        if (d->uev[k]) cudaEventDestroy(d->uev[k]);
+        if (d->ub[k]) cudaFreeHost(d->ub[k]);
+        d->uev[k] = nullptr;
+        d->ub[k] = nullptr;
+    }
+}
+
 template <class T, class Al>
 static spcg_status_t upload(spcg_device_t* d, const std::vector<T, Al>& v, const T** out) {
     void* p = nullptr;
-    spcg_status_t s = dev_malloc(d, v.size() * sizeof(T), &p);
+    const size_t bytes = v.size() * sizeof(T);
+    spcg_status_t s = dev_malloc(d, bytes, &p);
     if (s != SPCG_OK) return s;
-    if (!v.empty()) CK(cudaMemcpyAsync(p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice, d->stream));
+    if (bytes >= (4u << 20)) {
+        s = h2d_bounced(d, p, v.data(), bytes);
+        if (s != SPCG_OK) return s;
+    } else if (!v.empty()) {
+        CK(cudaMemcpyAsync(p, v.data(), bytes, cudaMemcpyHostToDevice, d->stream));
+    }
     *out = (const T*)p;
     return SPCG_OK;
 }
@@ -1735,6 +1785,7 @@ spcg_status_t spcg_dev_create(int device, void* stream, const spcg::Layouts& lay
         return SPCG_ERR_CUDA;
     }
     if (cudaStreamSynchronize(d->stream) != cudaSuccess) { spcg_dev_destroy(d); return SPCG_ERR_CUDA; }
+    release_bounce(d);
     *bytes = d->bytes;
     *out = d;
     return SPCG_OK;
@@ -1745,6 +1796,7 @@ void spcg_dev_destroy(spcg_device_t* d) {
     cudaSetDevice(d->device);
     cudaStreamSynchronize(d->stream);
     if (d->sc_host) cudaFreeHost(d->sc_host);
+    release_bounce(d);
     for (auto& a : d->allocs) {
         if (d->A.free) d->A.free(a.first, a.second, (void*)d->stream, d->A.ctx);
         else cudaFree(a.first);
