@@ -672,6 +672,49 @@ __device__ __forceinline__ void spmv_tma_stage(const int32_t* __restrict__ cs, c
     }
 }
 
+// Two stages at once: every gather of both is issued before the first is used (twice
+// the loads in flight per warp: the SpMV is gather-latency bound); the
+// values are re-read from shared memory at the FMA (registers for the gathers only).
+// Same accumulation order as two calls of spmv_tma_stage: bitwise the same w and (p, w).
+template <int WA>
+__device__ __forceinline__ void spmv_tma_pair(const int32_t* __restrict__ cs0, const double* __restrict__ vs0, int g0,
+                                              int64_t s0, const int32_t* __restrict__ cs1,
+                                              const double* __restrict__ vs1, int g1, int64_t s1,
+                                              const double* __restrict__ pin, double* __restrict__ wout, double& pw) {
+    constexpr int G = SPCG_SPMV_G;
+    const int lane = threadIdx.x & 31;
+    double gv0[G][WA], gv1[G][WA];
+#pragma unroll
+    for (int u = 0; u < G; ++u)
+#pragma unroll
+        for (int k = 0; k < WA; ++k) {
+            const int c0 = u < g0 ? cs0[(u * WA + k) * 32 + lane] : 0;
+            const int c1 = u < g1 ? cs1[(u * WA + k) * 32 + lane] : 0;
+            gv0[u][k] = u < g0 ? pin[c0] : 0.0;
+            gv1[u][k] = u < g1 ? pin[c1] : 0.0;
+        }
+#pragma unroll
+    for (int u = 0; u < G; ++u) {
+        if (u >= g0) break;
+        double acc = 0.0;
+#pragma unroll
+        for (int k = 0; k < WA; ++k) acc = fma(vs0[(u * WA + k) * 32 + lane], gv0[u][k], acc);
+        const int64_t row = (s0 + u) * 32 + lane;
+        wout[row] = acc;
+        pw = fma(pin[row], acc, pw);
+    }
+#pragma unroll
+    for (int u = 0; u < G; ++u) {
+        if (u >= g1) break;
+        double acc = 0.0;
+#pragma unroll
+        for (int k = 0; k < WA; ++k) acc = fma(vs1[(u * WA + k) * 32 + lane], gv1[u][k], acc);
+        const int64_t row = (s1 + u) * 32 + lane;
+        wout[row] = acc;
+        pw = fma(pin[row], acc, pw);
+    }
+}
+
 __device__ void chain_spmv_tma(const DevChain& D, const DevA& A, uint8_t* dyn, uint64_t* bars, unsigned& spq,
                                const double* __restrict__ pin, double* __restrict__ wout, double& pw, Scal* sc) {
     constexpr int G = SPCG_SPMV_G;
@@ -701,26 +744,47 @@ __device__ void chain_spmv_tma(const DevChain& D, const DevA& A, uint8_t* dyn, u
     long long t_all = SPCG_CHAIN_PROF ? clock64() : 0, t_wait = 0;
     if (lane == 0)
         for (int j = 0; j < min(NS, nst); ++j) issue(j);
-    for (int j = 0; j < nst; ++j) {
+    for (int j = 0; j < nst;) {
+        // narrow slices (WA <= 5: the registers of two stages' gathers fit) go two stages
+        // at a time
+        const bool two = WA <= 5 && j + 1 < nst;
         const unsigned u = spq + j;
         const long long tw = SPCG_CHAIN_PROF ? clock64() : 0;
         if (!warp_ok(mbar_wait(&bar[u % NS], (u / NS) & 1, sc))) return;
+        if (two && !warp_ok(mbar_wait(&bar[(u + 1) % NS], ((u + 1) / NS) & 1, sc))) return;
         if (SPCG_CHAIN_PROF) t_wait += clock64() - tw;
         const uint8_t* st = ring + (size_t)(u % NS) * D.sp_stage_bytes;
         const int32_t* cs = (const int32_t*)st;
         const double* vs = (const double*)(st + (size_t)G * WA * 128);
         const int64_t s = ((int64_t)j * NW + gw) * G;
         const int g = (int)(ns - s < (int64_t)G ? ns - s : (int64_t)G);
-        switch (WA) {
-            case 3: spmv_tma_stage<3>(cs, vs, g, s, pin, wout, pw); break;
-            case 4: spmv_tma_stage<4>(cs, vs, g, s, pin, wout, pw); break;
-            case 5: spmv_tma_stage<5>(cs, vs, g, s, pin, wout, pw); break;
-            case 6: spmv_tma_stage<6>(cs, vs, g, s, pin, wout, pw); break;
-            case 7: spmv_tma_stage<7>(cs, vs, g, s, pin, wout, pw); break;
-            default: spmv_tma_stage<8>(cs, vs, g, s, pin, wout, pw); break;
+        if (two) {
+            const uint8_t* st1 = ring + (size_t)((u + 1) % NS) * D.sp_stage_bytes;
+            const int32_t* cs1 = (const int32_t*)st1;
+            const double* vs1 = (const double*)(st1 + (size_t)G * WA * 128);
+            const int64_t s1 = ((int64_t)(j + 1) * NW + gw) * G;
+            const int g1 = (int)(ns - s1 < (int64_t)G ? ns - s1 : (int64_t)G);
+            switch (WA) {
+                case 3: spmv_tma_pair<3>(cs, vs, g, s, cs1, vs1, g1, s1, pin, wout, pw); break;
+                case 4: spmv_tma_pair<4>(cs, vs, g, s, cs1, vs1, g1, s1, pin, wout, pw); break;
+                default: spmv_tma_pair<5>(cs, vs, g, s, cs1, vs1, g1, s1, pin, wout, pw); break;
+            }
+        } else {
+            switch (WA) {
+                case 3: spmv_tma_stage<3>(cs, vs, g, s, pin, wout, pw); break;
+                case 4: spmv_tma_stage<4>(cs, vs, g, s, pin, wout, pw); break;
+                case 5: spmv_tma_stage<5>(cs, vs, g, s, pin, wout, pw); break;
+                case 6: spmv_tma_stage<6>(cs, vs, g, s, pin, wout, pw); break;
+                case 7: spmv_tma_stage<7>(cs, vs, g, s, pin, wout, pw); break;
+                default: spmv_tma_stage<8>(cs, vs, g, s, pin, wout, pw); break;
+            }
         }
         __syncwarp();
-        if (lane == 0 && j + NS < nst) issue(j + NS);
+        if (lane == 0) {
+            if (j + NS < nst) issue(j + NS);
+            if (two && j + 1 + NS < nst) issue(j + 1 + NS);
+        }
+        j += two ? 2 : 1;
     }
     spq += (unsigned)nst;
     if (SPCG_CHAIN_PROF && lane == 0 && g_chain_prof) {
